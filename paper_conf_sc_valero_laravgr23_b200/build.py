@@ -1,0 +1,69 @@
+"""Build libmrlbm.so in-tree with nvcc for sm_100a (no JIT, no torch extension)."""
+from __future__ import annotations
+
+import os
+import subprocess
+import sys
+from pathlib import Path
+
+PKG = Path(__file__).resolve().parent
+ROOT = PKG.parent
+CSRC = PKG / "csrc"
+LIB = PKG / "libmrlbm.so"
+SOURCES = [CSRC / "mrlbm.cu"]
+DEPS = SOURCES + [CSRC / "mrlbm_kernels.cuh", CSRC / "lattice.cuh", ROOT / "include" / "mrlbm.h"]
+
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+
+def nccl_dirs():
+    try:
+        import nvidia.nccl as nn  # the NCCL torch is built against (2.28.x)
+        base = Path(list(nn.__path__)[0])
+        inc, lib = base / "include", base / "lib"
+        if (inc / "nccl.h").exists():
+            return inc, lib
+    except Exception:
+        pass
+    return Path("/usr/include"), Path("/usr/lib/x86_64-linux-gnu")
+
+
+def nvcc():
+    for cand in (os.environ.get("NVCC"), "/usr/local/cuda/bin/nvcc", "nvcc"):
+        if cand and (Path(cand).exists() or cand == "nvcc"):
+            return cand
+    return "nvcc"
+
+
+def needs_build() -> bool:
+    if not LIB.exists():
+        return True
+    t = LIB.stat().st_mtime
+    return any(p.stat().st_mtime > t for p in DEPS)
+
+
+def build(force: bool = False, verbose: bool = False) -> Path:
+    if not force and not needs_build():
+        return LIB
+    inc, lib = nccl_dirs()
+    ncclso = "libnccl.so.2" if (lib / "libnccl.so.2").exists() else "libnccl.so"
+    tmp = LIB.with_suffix(f".{os.getpid()}.tmp.so")
+    cmd = [nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "--expt-relaxed-constexpr",
+           "-Xcompiler", "-fPIC", "-shared", "-o", str(tmp), *map(str, SOURCES),
+           f"-I{ROOT / 'include'}", f"-I{inc}", f"-L{lib}", f"-l:{ncclso}",
+           "-Xlinker", f"-rpath,{lib}"]
+    if verbose:
+        cmd += ["-Xptxas", "-v"]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        sys.stderr.write(r.stdout + r.stderr)
+        raise RuntimeError("nvcc failed building libmrlbm.so")
+    if verbose:
+        sys.stderr.write(r.stderr)
+    os.replace(tmp, LIB)
+    return LIB
+
+
+if __name__ == "__main__":
+    build(force="--force" in sys.argv, verbose="-v" in sys.argv)
+    print(LIB)

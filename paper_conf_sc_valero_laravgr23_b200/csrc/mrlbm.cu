@@ -1,0 +1,725 @@
+// mrlbm.cu -- host side of libmrlbm.so: the C ABI declared in include/mrlbm.h.
+//
+// Owns the device state (two SoA moment buffers, ping-pong, R7), builds the
+// TMA descriptors of both buffers, selects the template instance of the fused
+// step kernel (lattice x regularization x precision), batches steps into
+// CUDA graphs, and for nranks > 1 exchanges one boundary plane of moments per
+// step with each z-slab neighbour through NCCL send/recv on a communication
+// stream, overlapped with the interior update.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/mrlbm.h"
+#include "mrlbm_kernels.cuh"
+
+namespace {
+
+thread_local std::string g_last_error;
+
+mrlbm_status fail(mrlbm_status s, const std::string &msg)
+{
+    g_last_error = msg;
+    return s;
+}
+
+#define MR_CUDA(call)                                                                                \
+    do {                                                                                            \
+        cudaError_t e_ = (call);                                                                    \
+        if (e_ != cudaSuccess)                                                                      \
+            return fail(MRLBM_ERR_CUDA, std::string(#call) + ": " + cudaGetErrorString(e_));        \
+    } while (0)
+
+#define MR_NCCL(call)                                                                               \
+    do {                                                                                            \
+        ncclResult_t r_ = (call);                                                                   \
+        if (r_ != ncclSuccess) return fail(MRLBM_ERR_NCCL, std::string(#call) + ": " + ncclGetErrorString(r_)); \
+    } while (0)
+
+using mr::StepArgs;
+
+// ---------------------------------------------------------------- dispatch
+struct Variant {
+    int TA, TB, S, BW;
+    size_t smem;
+    void (*step)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t);
+    void (*set)(const double *, void *, mr::GridArgs, cudaStream_t);
+    void (*get)(const void *, double *, mr::GridArgs, cudaStream_t);
+    void (*pops)(const void *, double *, mr::GridArgs, double, cudaStream_t);
+    void (*finite)(const void *, mr::GridArgs, int *, cudaStream_t);
+    const void *kernel_fn;
+};
+
+inline int grid_for(long long n) { return (int)std::min<long long>((n + 255) / 256, 148LL * 16); }
+
+template <int LAT, bool REC, typename Real, int TA, int TB, int S> Variant make_variant()
+{
+    using L = mr::Lattice<LAT>;
+    using SM = mr::StepSmem<LAT, Real, TA, TB, S>;
+    Variant v;
+    v.TA = TA;
+    v.TB = TB;
+    v.S = S;
+    v.BW = SM::BW;
+    v.smem = SM::bytes;
+    v.kernel_fn = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S>;
+    v.step = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
+        mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S><<<grid, TA * TB, SM::bytes, st>>>(map, a);
+    };
+    v.set = [](const double *in, void *buf, mr::GridArgs g, cudaStream_t st) {
+        mr::set_moments_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
+            in, (Real *)buf, g);
+    };
+    v.get = [](const void *buf, double *out, mr::GridArgs g, cudaStream_t st) {
+        mr::get_moments_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
+            (const Real *)buf, out, g);
+    };
+    v.pops = [](const void *buf, double *out, mr::GridArgs g, double omega, cudaStream_t st) {
+        mr::populations_kernel<LAT, REC, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
+            (const Real *)buf, out, g, omega);
+    };
+    v.finite = [](const void *buf, mr::GridArgs g, int *flag, cudaStream_t st) {
+        mr::finite_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
+            (const Real *)buf, g, flag);
+    };
+    return v;
+}
+
+// Tile shapes: 2D one row of 128 threads (126 interior
+// nodes); 3D 32 x 8 threads (30 x 6 interior nodes) with a 3-deep TMA ring.
+template <int LAT, bool REC, typename Real> Variant pick()
+{
+    if constexpr (LAT == mr::LAT_D2Q9) return make_variant<LAT, REC, Real, 128, 1, 4>();
+    else return make_variant<LAT, REC, Real, 32, 8, 3>();
+}
+
+Variant select_variant(int lat, int reg, int prec)
+{
+    const bool R = reg == MRLBM_RECURSIVE;
+    const bool F = prec == MRLBM_FP32;
+#define MR_SEL(LAT)                                                                                 \
+    if (R) return F ? pick<LAT, true, float>() : pick<LAT, true, double>();                         \
+    else return F ? pick<LAT, false, float>() : pick<LAT, false, double>();
+    if (lat == MRLBM_D2Q9) { MR_SEL(mr::LAT_D2Q9) }
+    if (lat == MRLBM_D3Q19) { MR_SEL(mr::LAT_D3Q19) }
+    MR_SEL(mr::LAT_D3Q27)
+#undef MR_SEL
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode_fn()
+{
+    static EncodeTiledFn fn = nullptr;
+    if (!fn) {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = (EncodeTiledFn)p;
+    }
+    return fn;
+}
+
+} // namespace
+
+// ---------------------------------------------------------------- context
+struct mrlbm_ctx {
+    int lattice, reg, prec, D, M, Q, wbytes;
+    int64_t gn[3];        // global nx, ny, nz (nz = 1 in 2D)
+    int nA, nB, nC;       // local kernel extents
+    int cglobal, coff;    // global march extent, offset of this rank
+    int pitch, padA, padB;
+    long long mstride, pstride, origin; // origin: element offset of node (0,0) in a plane
+    size_t buf_bytes;
+    double tau, omega;
+    int rank = 0, nranks = 1, device = 0;
+    mrlbm_boundary bnd;   // physical faces (profiles re-pointed to device copies)
+    void *buf[2] = {nullptr, nullptr};
+    int cur = 0;
+    CUtensorMap tmap[2];
+    Variant var;
+    StepArgs base;        // template of the kernel arguments (src/dst filled per launch)
+    int tilesA, tilesB, seg_len, nseg;
+    cudaStream_t stream = nullptr, comm_stream = nullptr, cap_stream = nullptr;
+    bool own_stream = false;
+    cudaEvent_t ev_ready = nullptr, ev_comm = nullptr, ev_t0 = nullptr, ev_t1 = nullptr;
+    double *prof_dev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    double *io = nullptr;  // fp64 staging for set/get/populations
+    size_t io_bytes = 0;
+    int *flag = nullptr;
+    ncclComm_t comm = nullptr;
+    int nb_lo = -1, nb_hi = -1; // neighbour ranks along C (-1 none)
+    cudaGraphExec_t graph[2] = {nullptr, nullptr};
+    int graph_steps = 0;
+    int64_t kernels = 0;
+};
+
+namespace {
+
+// pointer to node (0,0) of plane 0 of buffer i
+void *node0(const mrlbm_ctx *h, int i) { return (char *)h->buf[i] + (size_t)h->origin * h->wbytes; }
+
+mr::GridArgs grid_args(const mrlbm_ctx *h)
+{
+    mr::GridArgs g;
+    g.nA = h->nA;
+    g.nB = h->nB;
+    g.nC = h->nC;
+    g.pitch = h->pitch;
+    g.mstride = h->mstride;
+    g.pstride = h->pstride;
+    return g;
+}
+
+// launch the fused kernel over owned layers [cb, ce) reading buf[src]
+void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st)
+{
+    if (ce <= cb) return;
+    StepArgs a = h->base;
+    a.src = node0(h, src);
+    a.dst = node0(h, 1 - src);
+    a.c_begin = cb;
+    a.c_end = ce;
+    const int span = ce - cb;
+    a.seg_len = std::min(h->seg_len, span);
+    const int nseg = (span + a.seg_len - 1) / a.seg_len;
+    dim3 grid(h->tilesA * h->tilesB, nseg);
+    h->var.step(h->tmap[src], a, grid, st);
+    h->kernels++;
+}
+
+mrlbm_status enqueue_one_step(mrlbm_ctx *h, cudaStream_t st)
+{
+    const int src = h->cur;
+    if (h->nranks == 1) {
+        launch_range(h, src, 0, h->nC, st);
+    } else {
+        // halo exchange of the boundary planes of the current state, overlapped
+        // with the interior layers [1, nC-1) that do not read the ghost planes
+        MR_CUDA(cudaEventRecord(h->ev_ready, st));
+        MR_CUDA(cudaStreamWaitEvent(h->comm_stream, h->ev_ready, 0));
+        char *base = (char *)h->buf[src];
+        const size_t plane = (size_t)h->pstride * h->wbytes;
+        const ncclDataType_t dt = h->prec == MRLBM_FP32 ? ncclFloat32 : ncclFloat64;
+        const size_t cnt = (size_t)h->pstride;
+        MR_NCCL(ncclGroupStart());
+        if (h->nb_hi >= 0) MR_NCCL(ncclSend(base + plane * h->nC, cnt, dt, h->nb_hi, h->comm, h->comm_stream));
+        if (h->nb_lo >= 0) MR_NCCL(ncclSend(base + plane * 1, cnt, dt, h->nb_lo, h->comm, h->comm_stream));
+        if (h->nb_lo >= 0) MR_NCCL(ncclRecv(base, cnt, dt, h->nb_lo, h->comm, h->comm_stream));
+        if (h->nb_hi >= 0) MR_NCCL(ncclRecv(base + plane * (h->nC + 1), cnt, dt, h->nb_hi, h->comm, h->comm_stream));
+        MR_NCCL(ncclGroupEnd());
+        MR_CUDA(cudaEventRecord(h->ev_comm, h->comm_stream));
+        launch_range(h, src, 1, h->nC - 1, st);
+        MR_CUDA(cudaStreamWaitEvent(st, h->ev_comm, 0));
+        launch_range(h, src, 0, 1, st);
+        launch_range(h, src, h->nC - 1, h->nC, st);
+    }
+    h->cur ^= 1;
+    MR_CUDA(cudaGetLastError());
+    return MRLBM_OK;
+}
+
+mrlbm_status ensure_io(mrlbm_ctx *h, size_t bytes)
+{
+    if (h->io_bytes >= bytes) return MRLBM_OK;
+    if (h->io) cudaFree(h->io);
+    h->io = nullptr;
+    h->io_bytes = 0;
+    if (cudaMalloc(&h->io, bytes) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(MRLBM_ERR_OUT_OF_MEMORY, "staging allocation failed");
+    }
+    h->io_bytes = bytes;
+    return MRLBM_OK;
+}
+
+bool is_wall(int k) { return k == MRLBM_WALL || k == MRLBM_MOVING_WALL; }
+bool is_open(int k) { return k == MRLBM_VELOCITY || k == MRLBM_PRESSURE; }
+
+} // namespace
+
+extern "C" {
+
+void mrlbm_default_options(mrlbm_options *o)
+{
+    if (!o) return;
+    memset(o, 0, sizeof(*o));
+    o->precision = MRLBM_FP64;
+    o->device = -1;
+    o->cuda_stream = nullptr;
+    o->rank = 0;
+    o->nranks = 1;
+    o->nccl_unique_id = nullptr;
+}
+
+const char *mrlbm_status_string(mrlbm_status s)
+{
+    switch (s) {
+    case MRLBM_OK: return "MRLBM_OK";
+    case MRLBM_ERR_INVALID_ARGUMENT: return "MRLBM_ERR_INVALID_ARGUMENT";
+    case MRLBM_ERR_UNSUPPORTED: return "MRLBM_ERR_UNSUPPORTED";
+    case MRLBM_ERR_OUT_OF_MEMORY: return "MRLBM_ERR_OUT_OF_MEMORY";
+    case MRLBM_ERR_CUDA: return "MRLBM_ERR_CUDA";
+    case MRLBM_ERR_NCCL: return "MRLBM_ERR_NCCL";
+    case MRLBM_ERR_NUMERICAL: return "MRLBM_ERR_NUMERICAL";
+    case MRLBM_ERR_BUFFER_SIZE: return "MRLBM_ERR_BUFFER_SIZE";
+    default: return "MRLBM_ERR_UNKNOWN";
+    }
+}
+
+const char *mrlbm_last_error(void) { return g_last_error.c_str(); }
+
+mrlbm_status mrlbm_nccl_unique_id(void *id128)
+{
+    if (!id128) return fail(MRLBM_ERR_INVALID_ARGUMENT, "id128 is NULL");
+    ncclUniqueId id;
+    MR_NCCL(ncclGetUniqueId(&id));
+    memcpy(id128, &id, sizeof(id));
+    return MRLBM_OK;
+}
+
+// Slab partition of the march axis: remainder spread over the first ranks.
+// Pure host arithmetic (no CUDA), exported for the distributed tests.
+mrlbm_status mrlbm_partition(int64_t n, int nranks, int rank, int64_t *n_local, int64_t *offset)
+{
+    if (nranks < 1 || rank < 0 || rank >= nranks || n < 1) return fail(MRLBM_ERR_INVALID_ARGUMENT, "bad partition");
+    const int64_t q = n / nranks, r = n % nranks;
+    *n_local = q + (rank < r ? 1 : 0);
+    *offset = rank * q + std::min<int64_t>(rank, r);
+    return MRLBM_OK;
+}
+
+// Validation of the create arguments without touching a GPU (exported for
+// the host-logic tests).  Returns the status mrlbm_create would return.
+mrlbm_status mrlbm_validate(mrlbm_lattice lattice, int64_t nx, int64_t ny, int64_t nz, double tau,
+                            mrlbm_regularization reg, const mrlbm_boundary *bnd, int nranks)
+{
+    if (lattice < MRLBM_D2Q9 || lattice > MRLBM_D3Q27) return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown lattice");
+    if (reg != MRLBM_PROJECTIVE && reg != MRLBM_RECURSIVE) return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown regularization");
+    if (!(tau > 0.5) || !std::isfinite(tau)) return fail(MRLBM_ERR_INVALID_ARGUMENT, "tau must be > 1/2 (eq 5)");
+    const int D = lattice == MRLBM_D2Q9 ? 2 : 3;
+    if (nx < 2 || ny < 2) return fail(MRLBM_ERR_INVALID_ARGUMENT, "nx, ny must be >= 2");
+    if (D == 2 && nz != 1) return fail(MRLBM_ERR_INVALID_ARGUMENT, "D2Q9 requires nz == 1");
+    if (D == 3 && nz < 2) return fail(MRLBM_ERR_INVALID_ARGUMENT, "nz must be >= 2");
+    if (nx > (1 << 30) || ny > (1 << 30) || nz > (1 << 30)) return fail(MRLBM_ERR_INVALID_ARGUMENT, "extent too large");
+    if (nranks < 1) return fail(MRLBM_ERR_INVALID_ARGUMENT, "nranks < 1");
+    const int64_t nmarch = D == 3 ? nz : ny;
+    if (nmarch / nranks < 2) return fail(MRLBM_ERR_INVALID_ARGUMENT, "each rank needs >= 2 layers along the slab axis");
+    if (!bnd) return MRLBM_OK;
+    for (int F = 0; F < 2 * D; F++) {
+        const int k = bnd->face[F].kind;
+        if (k < MRLBM_PERIODIC || k > MRLBM_PRESSURE) return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown face kind");
+    }
+    for (int ax = 0; ax < D; ax++) {
+        const bool p0 = bnd->face[2 * ax].kind == MRLBM_PERIODIC, p1 = bnd->face[2 * ax + 1].kind == MRLBM_PERIODIC;
+        if (p0 != p1) return fail(MRLBM_ERR_INVALID_ARGUMENT, "periodic on only one face of an axis");
+    }
+    for (int F = 0; F < 2 * D; F++) {
+        const mrlbm_face &f = bnd->face[F];
+        if (f.kind == MRLBM_MOVING_WALL && f.u[F / 2] != 0.0)
+            return fail(MRLBM_ERR_INVALID_ARGUMENT, "moving-wall velocity must be tangential");
+        if (f.kind == MRLBM_MOVING_WALL && D == 2 && f.u[2] != 0.0)
+            return fail(MRLBM_ERR_INVALID_ARGUMENT, "2D moving-wall velocity has a z component");
+        if (f.kind == MRLBM_PRESSURE && !(f.rho > 0)) return fail(MRLBM_ERR_INVALID_ARGUMENT, "pressure face needs rho > 0");
+    }
+    const int march = D == 3 ? 2 : 1;
+    if (is_open(bnd->face[2 * march].kind) || is_open(bnd->face[2 * march + 1].kind))
+        return fail(MRLBM_ERR_UNSUPPORTED, "open faces on the marching/slab axis are not supported");
+    if (D == 3) {
+        const bool ox = is_open(bnd->face[0].kind) || is_open(bnd->face[1].kind);
+        const bool oy = is_open(bnd->face[2].kind) || is_open(bnd->face[3].kind);
+        if (ox && oy) return fail(MRLBM_ERR_UNSUPPORTED, "open faces sharing an edge");
+    }
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64_t ny, int64_t nz, double tau,
+                          mrlbm_regularization reg, const mrlbm_boundary *boundary, const mrlbm_options *opt)
+{
+    if (!out) return fail(MRLBM_ERR_INVALID_ARGUMENT, "out is NULL");
+    *out = nullptr;
+    mrlbm_options o;
+    mrlbm_default_options(&o);
+    if (opt) o = *opt;
+    if (o.precision != MRLBM_FP64 && o.precision != MRLBM_FP32) return fail(MRLBM_ERR_INVALID_ARGUMENT, "precision");
+    mrlbm_status st = mrlbm_validate(lattice, nx, ny, nz, tau, reg, boundary, o.nranks);
+    if (st) return st;
+    if (o.nranks > 1 && !o.nccl_unique_id) return fail(MRLBM_ERR_INVALID_ARGUMENT, "nranks > 1 needs nccl_unique_id");
+    if (o.rank < 0 || o.rank >= o.nranks) return fail(MRLBM_ERR_INVALID_ARGUMENT, "rank out of range");
+
+    EncodeTiledFn encode = get_encode_fn();
+    if (o.device >= 0) MR_CUDA(cudaSetDevice(o.device));
+    int dev = 0;
+    MR_CUDA(cudaGetDevice(&dev));
+    if (!encode) return fail(MRLBM_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+
+    mrlbm_ctx *h = new mrlbm_ctx();
+    h->device = dev;
+    h->lattice = lattice;
+    h->reg = reg;
+    h->prec = o.precision;
+    h->D = lattice == MRLBM_D2Q9 ? 2 : 3;
+    h->M = h->D == 2 ? 6 : 10;
+    h->Q = lattice == MRLBM_D2Q9 ? 9 : (lattice == MRLBM_D3Q19 ? 19 : 27);
+    h->wbytes = o.precision == MRLBM_FP32 ? 4 : 8;
+    h->gn[0] = nx;
+    h->gn[1] = ny;
+    h->gn[2] = h->D == 2 ? 1 : nz;
+    h->tau = tau;
+    h->omega = 1.0 - 1.0 / tau;
+    h->rank = o.rank;
+    h->nranks = o.nranks;
+    if (boundary) h->bnd = *boundary;
+    else memset(&h->bnd, 0, sizeof(h->bnd)); // all periodic
+
+    // kernel axes: A = x, B = y (3D) / 1 (2D), C = z (3D) / y (2D)
+    h->nA = (int)nx;
+    h->nB = h->D == 3 ? (int)ny : 1;
+    h->cglobal = (int)(h->D == 3 ? nz : ny);
+    int64_t nloc, off;
+    mrlbm_partition(h->cglobal, o.nranks, o.rank, &nloc, &off);
+    h->nC = (int)nloc;
+    h->coff = (int)off;
+    // Storage: each A-row starts with padA elements (16 B) and, in 3D, each
+    // moment plane with one pad row, so that every TMA box origin (tile origin
+    // minus the halo) is a non-negative coordinate.  Rows are 32-B aligned.
+    h->padA = 16 / h->wbytes;
+    h->padB = h->D == 3 ? 1 : 0;
+    const int align = 32 / h->wbytes;
+    h->pitch = (h->padA + h->nA + align - 1) / align * align;
+    h->mstride = (long long)(h->padB + h->nB) * h->pitch;
+    h->origin = (long long)h->padB * h->pitch + h->padA;
+    h->pstride = (long long)h->M * h->mstride;
+    h->buf_bytes = (size_t)(h->nC + 2) * h->pstride * h->wbytes;
+
+    auto cleanup_fail = [&](mrlbm_status s) {
+        mrlbm_destroy(h);
+        return s;
+    };
+
+    if (o.cuda_stream) {
+        h->stream = (cudaStream_t)o.cuda_stream;
+    } else {
+        if (cudaStreamCreateWithFlags(&h->stream, cudaStreamNonBlocking) != cudaSuccess)
+            return cleanup_fail(fail(MRLBM_ERR_CUDA, "stream create"));
+        h->own_stream = true;
+    }
+    if (cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&h->ev_ready, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&h->ev_comm, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreate(&h->ev_t0) != cudaSuccess || cudaEventCreate(&h->ev_t1) != cudaSuccess)
+        return cleanup_fail(fail(MRLBM_ERR_CUDA, "stream/event create"));
+
+    for (int i = 0; i < 2; i++) {
+        if (cudaMalloc(&h->buf[i], h->buf_bytes) != cudaSuccess) {
+            cudaGetLastError();
+            return cleanup_fail(fail(MRLBM_ERR_OUT_OF_MEMORY, "state allocation failed"));
+        }
+        if (cudaMemsetAsync(h->buf[i], 0, h->buf_bytes, h->stream) != cudaSuccess)
+            return cleanup_fail(fail(MRLBM_ERR_CUDA, "memset"));
+    }
+    if (cudaMalloc(&h->flag, sizeof(int)) != cudaSuccess) return cleanup_fail(fail(MRLBM_ERR_OUT_OF_MEMORY, "flag"));
+
+    // velocity profiles -> device
+    for (int F = 0; F < 2 * h->D; F++) {
+        mrlbm_face &f = h->bnd.face[F];
+        if (f.kind == MRLBM_VELOCITY && f.u_profile) {
+            const int ax = F / 2;
+            const size_t nodes = (size_t)(nx * ny * h->gn[2]) / (size_t)h->gn[ax];
+            const size_t bytes = nodes * h->D * sizeof(double);
+            if (cudaMalloc(&h->prof_dev[F], bytes) != cudaSuccess) return cleanup_fail(fail(MRLBM_ERR_OUT_OF_MEMORY, "profile"));
+            if (cudaMemcpy(h->prof_dev[F], f.u_profile, bytes, cudaMemcpyHostToDevice) != cudaSuccess)
+                return cleanup_fail(fail(MRLBM_ERR_CUDA, "profile copy"));
+        }
+        f.u_profile = nullptr;
+    }
+
+    h->var = select_variant(lattice, reg, o.precision);
+    if (cudaFuncSetAttribute(h->var.kernel_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)h->var.smem) !=
+        cudaSuccess)
+        return cleanup_fail(fail(MRLBM_ERR_CUDA, "smem attribute"));
+
+    // TMA descriptors: tensor {nA, nB, M, nC + 2} of the [plane][m][b][a] layout
+    for (int i = 0; i < 2; i++) {
+        cuuint64_t dims[4] = {(cuuint64_t)(h->padA + h->nA), (cuuint64_t)(h->padB + h->nB), (cuuint64_t)h->M,
+                              (cuuint64_t)(h->nC + 2)};
+        cuuint64_t strides[3] = {(cuuint64_t)h->pitch * h->wbytes, (cuuint64_t)h->mstride * h->wbytes,
+                                 (cuuint64_t)h->pstride * h->wbytes};
+        cuuint32_t box[4] = {(cuuint32_t)h->var.BW, (cuuint32_t)h->var.TB, (cuuint32_t)h->M, 1};
+        cuuint32_t estr[4] = {1, 1, 1, 1};
+        CUresult r = encode(&h->tmap[i], h->prec == MRLBM_FP32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT64,
+                            4, h->buf[i], dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                            CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (r != CUDA_SUCCESS) return cleanup_fail(fail(MRLBM_ERR_CUDA, "cuTensorMapEncodeTiled failed: " + std::to_string((int)r)));
+    }
+
+    // kernel argument template: physical faces -> kernel faces A-,A+,B-,B+,C-,C+
+    StepArgs &a = h->base;
+    memset(&a, 0, sizeof(a));
+    a.nA = h->nA;
+    a.nB = h->nB;
+    a.nC = h->nC;
+    a.pitch = h->pitch;
+    a.padA = h->padA;
+    a.padB = h->padB;
+    a.mstride = h->mstride;
+    a.pstride = h->pstride;
+    a.omega = h->omega;
+    a.c_offset = h->coff;
+    const int phys[6] = {0, 1, h->D == 3 ? 2 : -1, h->D == 3 ? 3 : -1, h->D == 3 ? 4 : 2, h->D == 3 ? 5 : 3};
+    for (int K = 0; K < 6; K++) {
+        if (phys[K] < 0) {
+            a.kind[K] = mr::BC_PERIODIC;
+            continue;
+        }
+        const mrlbm_face &f = h->bnd.face[phys[K]];
+        a.kind[K] = f.kind;
+        for (int q = 0; q < 3; q++) a.uw[K][q] = f.kind == MRLBM_MOVING_WALL ? f.u[q] : 0.0;
+        if (K < 4) {
+            a.open_drho[K] = f.rho - 1.0;
+            for (int q = 0; q < 3; q++) a.open_u[K][q] = f.u[q];
+            a.open_prof[K] = h->prof_dev[phys[K]];
+        }
+    }
+    const bool perC = a.kind[4] == mr::BC_PERIODIC;
+    if (h->nranks == 1) {
+        a.wrapC = perC ? 1 : 0;
+        a.lo_nb = a.hi_nb = perC ? 1 : 0;
+    } else {
+        a.wrapC = 0;
+        h->nb_lo = (h->rank > 0) ? h->rank - 1 : (perC ? h->nranks - 1 : -1);
+        h->nb_hi = (h->rank < h->nranks - 1) ? h->rank + 1 : (perC ? 0 : -1);
+        a.lo_nb = h->nb_lo >= 0;
+        a.hi_nb = h->nb_hi >= 0;
+        if (a.lo_nb) a.kind[4] = mr::BC_PERIODIC; // interior cut: neighbour data in the ghost plane
+        if (a.hi_nb) a.kind[5] = mr::BC_PERIODIC;
+    }
+    const int TA = h->var.TA, TB = h->var.TB;
+    h->tilesA = (h->nA + TA - 3) / (TA - 2);
+    h->tilesB = h->D == 3 ? (h->nB + TB - 3) / (TB - 2) : 1;
+    a.tilesA = h->tilesA;
+    // segments along C: aim for >= 8 resident waves of CTAs, segments >= 8 layers
+    {
+        const long long tiles = (long long)h->tilesA * h->tilesB;
+        const long long target = 148LL * 8;
+        long long nseg = std::max<long long>(1, target / std::max<long long>(1, tiles));
+        long long seg = (h->nC + nseg - 1) / nseg;
+        seg = std::max<long long>(seg, std::min<long long>(8, h->nC));
+        h->seg_len = (int)seg;
+        h->nseg = (int)((h->nC + seg - 1) / seg);
+    }
+
+    if (h->nranks > 1) {
+        if (cudaStreamCreateWithFlags(&h->comm_stream, cudaStreamNonBlocking) != cudaSuccess)
+            return cleanup_fail(fail(MRLBM_ERR_CUDA, "comm stream"));
+        ncclUniqueId id;
+        memcpy(&id, o.nccl_unique_id, sizeof(id));
+        ncclResult_t r = ncclCommInitRank(&h->comm, h->nranks, id, h->rank);
+        if (r != ncclSuccess) return cleanup_fail(fail(MRLBM_ERR_NCCL, std::string("ncclCommInitRank: ") + ncclGetErrorString(r)));
+    }
+
+    // rest state: rho = 1 (stored rho - 1 = 0), u = 0, Pi = 0 -> zeros (done by memset)
+    if (cudaStreamSynchronize(h->stream) != cudaSuccess) return cleanup_fail(fail(MRLBM_ERR_CUDA, "sync"));
+    *out = h;
+    return MRLBM_OK;
+}
+
+void mrlbm_destroy(mrlbm_t h)
+{
+    if (!h) return;
+    if (h->stream) cudaStreamSynchronize(h->stream);
+    if (h->comm) ncclCommDestroy(h->comm);
+    for (int i = 0; i < 2; i++)
+        if (h->graph[i]) cudaGraphExecDestroy(h->graph[i]);
+    for (int i = 0; i < 2; i++)
+        if (h->buf[i]) cudaFree(h->buf[i]);
+    for (int F = 0; F < 6; F++)
+        if (h->prof_dev[F]) cudaFree(h->prof_dev[F]);
+    if (h->io) cudaFree(h->io);
+    if (h->flag) cudaFree(h->flag);
+    if (h->ev_ready) cudaEventDestroy(h->ev_ready);
+    if (h->ev_comm) cudaEventDestroy(h->ev_comm);
+    if (h->ev_t0) cudaEventDestroy(h->ev_t0);
+    if (h->ev_t1) cudaEventDestroy(h->ev_t1);
+    if (h->comm_stream) cudaStreamDestroy(h->comm_stream);
+    if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
+    if (h->own_stream && h->stream) cudaStreamDestroy(h->stream);
+    delete h;
+}
+
+static int64_t local_nodes(const mrlbm_ctx *h) { return (int64_t)h->nA * h->nB * h->nC; }
+
+mrlbm_status mrlbm_set_moments_device(mrlbm_t h, const double *src_dev, int64_t count)
+{
+    if (!h || !src_dev) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
+    if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
+    h->var.set(src_dev, node0(h, h->cur), grid_args(h), h->stream);
+    MR_CUDA(cudaGetLastError());
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_get_moments_device(mrlbm_t h, double *dst_dev, int64_t count)
+{
+    if (!h || !dst_dev) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
+    if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
+    h->var.get(node0(h, h->cur), dst_dev, grid_args(h), h->stream);
+    MR_CUDA(cudaGetLastError());
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_set_moments(mrlbm_t h, const double *src, int64_t count)
+{
+    if (!h || !src) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
+    if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
+    mrlbm_status s = ensure_io(h, (size_t)count * sizeof(double));
+    if (s) return s;
+    MR_CUDA(cudaMemcpyAsync(h->io, src, (size_t)count * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+    s = mrlbm_set_moments_device(h, h->io, count);
+    if (s) return s;
+    MR_CUDA(cudaStreamSynchronize(h->stream));
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_get_moments(mrlbm_t h, double *dst, int64_t count)
+{
+    if (!h || !dst) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
+    if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
+    mrlbm_status s = ensure_io(h, (size_t)count * sizeof(double));
+    if (s) return s;
+    s = mrlbm_get_moments_device(h, h->io, count);
+    if (s) return s;
+    MR_CUDA(cudaMemcpyAsync(dst, h->io, (size_t)count * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    MR_CUDA(cudaStreamSynchronize(h->stream));
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_get_populations(mrlbm_t h, double *dst, int64_t count)
+{
+    if (!h || !dst) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
+    if (count != (int64_t)h->Q * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != Q * N_local");
+    mrlbm_status s = ensure_io(h, (size_t)count * sizeof(double));
+    if (s) return s;
+    h->var.pops(node0(h, h->cur), h->io, grid_args(h), h->omega, h->stream);
+    MR_CUDA(cudaGetLastError());
+    MR_CUDA(cudaMemcpyAsync(dst, h->io, (size_t)count * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    MR_CUDA(cudaStreamSynchronize(h->stream));
+    return MRLBM_OK;
+}
+
+static const int kGraphSteps = 32; // even: a replay returns the ping-pong parity
+
+mrlbm_status mrlbm_step(mrlbm_t h, int64_t n)
+{
+    if (!h || n < 0) return fail(MRLBM_ERR_INVALID_ARGUMENT, "bad step count");
+    // Batches of kGraphSteps single-rank steps are replayed from a captured graph.
+    while (h->nranks == 1 && n >= kGraphSteps) {
+        const int par = h->cur;
+        if (!h->graph[par]) {
+            cudaGraph_t g;
+            MR_CUDA(cudaStreamBeginCapture(h->cap_stream, cudaStreamCaptureModeThreadLocal));
+            const int64_t k0 = h->kernels;
+            for (int i = 0; i < kGraphSteps; i++) {
+                mrlbm_status s = enqueue_one_step(h, h->cap_stream);
+                if (s) {
+                    cudaStreamEndCapture(h->cap_stream, &g);
+                    return s;
+                }
+            }
+            h->graph_steps = (int)(h->kernels - k0);
+            h->kernels = k0;
+            MR_CUDA(cudaStreamEndCapture(h->cap_stream, &g));
+            MR_CUDA(cudaGraphInstantiate(&h->graph[par], g, 0));
+            cudaGraphDestroy(g);
+            h->cur = par; // capture only recorded the steps
+        }
+        MR_CUDA(cudaGraphLaunch(h->graph[par], h->stream));
+        h->kernels += h->graph_steps;
+        n -= kGraphSteps;
+    }
+    for (int64_t i = 0; i < n; i++) {
+        mrlbm_status s = enqueue_one_step(h, h->stream);
+        if (s) return s;
+    }
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_sync(mrlbm_t h)
+{
+    if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
+    MR_CUDA(cudaStreamSynchronize(h->stream));
+    if (h->comm_stream) MR_CUDA(cudaStreamSynchronize(h->comm_stream));
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_check_finite(mrlbm_t h)
+{
+    if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
+    MR_CUDA(cudaMemsetAsync(h->flag, 0, sizeof(int), h->stream));
+    h->var.finite(node0(h, h->cur), grid_args(h), h->flag, h->stream);
+    int v = 0;
+    MR_CUDA(cudaMemcpyAsync(&v, h->flag, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
+    MR_CUDA(cudaStreamSynchronize(h->stream));
+    return v ? fail(MRLBM_ERR_NUMERICAL, "non-finite moment in the state") : MRLBM_OK;
+}
+
+mrlbm_status mrlbm_query(mrlbm_t h, int64_t *M, int64_t *Q, int64_t *n_local, int64_t *offset, int64_t *bytes)
+{
+    if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
+    if (M) *M = h->M;
+    if (Q) *Q = h->Q;
+    if (n_local) *n_local = h->nC;
+    if (offset) *offset = h->coff;
+    if (bytes) *bytes = (int64_t)(2 * h->buf_bytes);
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_launch_count(mrlbm_t h, int64_t *kernels)
+{
+    if (!h || !kernels) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
+    *kernels = h->kernels;
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_time_steps(mrlbm_t h, int64_t n, double *ms_per_step)
+{
+    if (!h || !ms_per_step || n < 1) return fail(MRLBM_ERR_INVALID_ARGUMENT, "bad argument");
+    MR_CUDA(cudaEventRecord(h->ev_t0, h->stream));
+    mrlbm_status s = mrlbm_step(h, n);
+    if (s) return s;
+    MR_CUDA(cudaEventRecord(h->ev_t1, h->stream));
+    MR_CUDA(cudaEventSynchronize(h->ev_t1));
+    float ms = 0.f;
+    MR_CUDA(cudaEventElapsedTime(&ms, h->ev_t0, h->ev_t1));
+    *ms_per_step = ms / (double)n;
+    return MRLBM_OK;
+}
+
+// Internal layout description, for the bench's roofline bookkeeping and tests:
+// tile shape, segment length and grid of the fused kernel.
+mrlbm_status mrlbm_kernel_config(mrlbm_t h, int *TA, int *TB, int *S, int *seg_len, int *grid_x, int *grid_y,
+                                 int64_t *smem_bytes)
+{
+    if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
+    if (TA) *TA = h->var.TA;
+    if (TB) *TB = h->var.TB;
+    if (S) *S = h->var.S;
+    if (seg_len) *seg_len = h->seg_len;
+    if (grid_x) *grid_x = h->tilesA * h->tilesB;
+    if (grid_y) *grid_y = h->nseg;
+    if (smem_bytes) *smem_bytes = (int64_t)h->var.smem;
+    return MRLBM_OK;
+}
+
+} // extern "C"

@@ -1,0 +1,607 @@
+// mrlbm_kernels.cuh -- the fused sm_100a MR-LBM timestep and its helpers.
+//
+// One launch = one timestep of the moment representation (Alg. 2,
+// P:L185-261): read the moments (rho, u, Pi) of a tile, collide in moment
+// space (eq 10; eqs 12-13 for recursive), reconstruct the post-collision
+// populations (eq 11 / eq 14), stream them (eq 7) across the CTA through
+// shared memory with a one-node halo, apply the boundary
+// treatment, recompute the moments of the completed layer (eqs 1-3,
+// P:L259) and write them back.  Only moments touch HBM.
+//
+// B200 design: a CTA owns a (TA-2) x (TB-2) in-plane
+// tile (2D: TA-2 x 1) and sweeps a segment of layers along the marching
+// axis C.  Per layer a TMA box {TA, TB, M, 1} (tile + halo ring, all M
+// moment planes) lands in an S-deep shared-memory ring guarded by mbarriers;
+// in-plane moving populations are exchanged through one shared-memory plane;
+// populations moving along C never leave the thread: they are accumulated
+// into rolling per-layer moment accumulators (layers c-1, c, c+1) held in
+// registers, which replaces the paper's (z_t + 2)-layer shared population
+// array.  The state is stored shifted (rho - 1, populations f - w_i) for
+// precision (R16).
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "lattice.cuh"
+
+namespace mr {
+
+enum { BC_PERIODIC = 0, BC_WALL = 1, BC_MOVING = 2, BC_VELOCITY = 3, BC_PRESSURE = 4 };
+
+// Kernel-axis faces: 0 A-, 1 A+, 2 B-, 3 B+, 4 C-, 5 C+.
+struct StepArgs {
+    const void *src;        // node (0,0) of plane 0 (low ghost plane) of the source buffer
+    void *dst;              // same for the destination buffer
+    int padA, padB;         // storage pad before node 0 along A / B (TMA box origins must be >= 0)
+    int nA, nB, nC;         // local extents (nB = 1 in 2D)
+    int pitch;              // elements per A-row
+    long long mstride;      // elements between moment planes = nB * pitch
+    long long pstride;      // elements between layers         = M * nB * pitch
+    int c_begin, c_end;     // owned layers updated by this launch
+    int seg_len;            // layers per CTA segment
+    int tilesA;             // tiles along A (grid.x = tilesA * tilesB)
+    int lo_nb, hi_nb;       // 1 if layer -1 / nC exists (periodic wrap or ghost plane)
+    int wrapC;              // 1: layer c lives in plane wrap(c)+1 (single-rank periodic C)
+    int c_offset;           // global index of local layer 0 (profiles)
+    int kind[6];            // face kinds (C faces: WALL/MOVING only at this rank's global ends)
+    double uw[6][3];        // wall velocities (physical x, y, z)
+    double open_drho[4];    // PRESSURE faces: rho - 1
+    double open_u[4][3];    // VELOCITY faces: uniform velocity
+    const double *open_prof[4]; // VELOCITY faces: optional [face nodes][D] (global)
+    double omega;           // 1 - 1/tau
+};
+
+// ------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void *p)
+{
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count)
+{
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_barrier_init()
+{
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t *bar, uint32_t bytes)
+{
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
+{
+    uint32_t addr = smem_u32(bar);
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(addr),
+        "r"(parity)
+        : "memory");
+}
+__device__ __forceinline__ void tma_load_4d(void *dst, const CUtensorMap *map, uint64_t *bar, int c0, int c1,
+                                            int c2, int c3)
+{
+    asm volatile(
+        "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], "
+        "[%2];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+        : "memory");
+}
+__device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map)
+{
+    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+
+// ------------------------------------------------------------ node algebra
+// Collided, scaled Hermite coefficients A'_h of one node (eqs 10, 12, 13 and
+// their orders-5/6 extension for D3Q27; recursive a^neq from the pair-sum
+// closed form of Malaspinas' recursion, R8):
+//   n = 0: rho - 1 (shifted zeroth moment)     n = 1: rho u_a
+//   n = 2: omega Pi_ab + (1 - omega) rho u_a u_b           (= Pi*, eq 10)
+//   n > 2: rho prod u + omega sum_{p<q} Pneq_{a_p a_q} prod_{k != p,q} u_{a_k}
+// each times hscale(h).
+template <int LAT, bool REC, typename Real>
+__device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M], Real omega,
+                                               Real (&A)[Basis<LAT, REC>::NH])
+{
+    using L = Lattice<LAT>;
+    using B = Basis<LAT, REC>;
+    constexpr int D = L::D;
+    const Real drho = m[0];
+    const Real rho = Real(1) + drho;
+    Real u[3];
+    u[0] = m[1];
+    u[1] = m[2];
+    u[2] = (D == 3) ? m[3] : Real(0);
+    const Real omc = Real(1) - omega;
+    Real Pn[3][3]; // Pi^neq (eq 8 in moment form: Pi - rho u u)
+    if constexpr (REC) {
+#pragma unroll
+        for (int a = 0; a < D; a++)
+#pragma unroll
+            for (int b = a; b < D; b++) {
+                Pn[a][b] = m[pslot<D>(a, b)] - rho * u[a] * u[b];
+                Pn[b][a] = Pn[a][b];
+            }
+    }
+    static_for<0, B::NH>([&](auto hk) {
+        constexpr int k = decltype(hk)::value;
+        constexpr int h0 = B::h[k][0], h1 = B::h[k][1], h2 = B::h[k][2];
+        constexpr int n = h0 + h1 + h2;
+        constexpr Real sc = Real(hscale(h0, h1, h2));
+        // axis labels of the component
+        constexpr int i0 = (h0 > 0) ? 0 : ((h1 > 0) ? 1 : 2);
+        Real val;
+        if constexpr (n == 0) {
+            val = drho;
+        } else if constexpr (n == 1) {
+            val = rho * u[i0];
+        } else if constexpr (n == 2) {
+            constexpr int i1 = (h0 == 2) ? 0 : ((h0 == 1) ? ((h1 > 0) ? 1 : 2) : ((h1 == 2) ? 1 : 2));
+            val = omega * m[pslot<D>(i0, i1)] + omc * rho * u[i0] * u[i1];
+        } else {
+            constexpr int idx[6] = {
+                0 < h0 ? 0 : (0 < h0 + h1 ? 1 : 2), 1 < h0 ? 0 : (1 < h0 + h1 ? 1 : 2),
+                2 < h0 ? 0 : (2 < h0 + h1 ? 1 : 2), 3 < h0 ? 0 : (3 < h0 + h1 ? 1 : 2),
+                4 < h0 ? 0 : (4 < h0 + h1 ? 1 : 2), 5 < h0 ? 0 : (5 < h0 + h1 ? 1 : 2)};
+            Real aeq = rho;
+#pragma unroll
+            for (int t = 0; t < n; t++) aeq *= u[idx[t]];
+            Real aneq = Real(0);
+#pragma unroll
+            for (int p = 0; p < n; p++)
+#pragma unroll
+                for (int q = p + 1; q < n; q++) {
+                    Real t = Pn[idx[p]][idx[q]];
+#pragma unroll
+                    for (int r = 0; r < n; r++)
+                        if (r != p && r != q) t *= u[idx[r]];
+                    aneq += t;
+                }
+            val = aeq + omega * aneq;
+        }
+        A[k] = val * sc;
+    });
+}
+
+// Multiply-accumulate by a small compile-time integer.
+template <int K, typename Real> __device__ __forceinline__ void acc_int(Real &s, Real v)
+{
+    if constexpr (K == 1) s += v;
+    else if constexpr (K == -1) s -= v;
+    else if constexpr (K != 0) s = fma(Real(K), v, s);
+}
+
+// Shifted post-collision populations f~*_i = f*_i - w_i (eq 11 / eq 14):
+// f~*_i = w_i sum_h He'_h(c_i) A'_h, evaluated for i and opp(i) together from
+// the even (E) and odd (O) parts of the basis: f_i = w(E+O), f_opp = w(E-O).
+template <int LAT, bool REC, typename Real>
+__device__ __forceinline__ void reconstruct(const Real (&A)[Basis<LAT, REC>::NH], Real (&f)[Lattice<LAT>::Q])
+{
+    using L = Lattice<LAT>;
+    using B = Basis<LAT, REC>;
+    static_for<0, L::HALF + 1>([&](auto ik) {
+        constexpr int i = decltype(ik)::value;
+        Real E = Real(0), O = Real(0);
+        static_for<0, B::NH>([&](auto hk) {
+            constexpr int k = decltype(hk)::value;
+            constexpr int h0 = B::h[k][0], h1 = B::h[k][1], h2 = B::h[k][2];
+            constexpr int he = he1s(h0, L::c[i][0]) * he1s(h1, L::c[i][1]) * he1s(h2, L::c[i][2]);
+            constexpr bool odd = ((h0 == 1) + (h1 == 1) + (h2 == 1)) % 2 == 1;
+            if constexpr (odd) acc_int<he>(O, A[k]);
+            else acc_int<he>(E, A[k]);
+        });
+        constexpr Real w = Real(L::w[i]);
+        if constexpr (i == 0) {
+            f[0] = w * E;
+        } else {
+            f[i] = w * (E + O);
+            f[i + L::HALF] = w * (E - O);
+        }
+    });
+}
+
+// Accumulate one arriving shifted population v with velocity c_k into the
+// raw moment accumulators (sum f~, sum c f~, sum c c f~).
+template <class L, int k, typename Real> __device__ __forceinline__ void accum(Real (&acc)[L::M], Real v)
+{
+    constexpr int D = L::D;
+    acc[0] += v;
+    static_for<0, D>([&](auto ak) {
+        constexpr int a = decltype(ak)::value;
+        acc_int<L::c[k][a]>(acc[1 + a], v);
+        static_for<a, D>([&](auto bk) {
+            constexpr int b = decltype(bk)::value;
+            acc_int<L::c[k][a] * L::c[k][b]>(acc[pslot<D>(a, b)], v);
+        });
+    });
+}
+
+// ------------------------------------------------------------ step kernel
+template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
+    using L = Lattice<LAT>;
+    static constexpr int NT = TA * TB;
+    // TMA box rows must start on a 16-byte boundary: the box starts at the
+    // window origin rounded down to AL elements and is BW elements wide.
+    static constexpr int AL = 16 / int(sizeof(Real));
+    static constexpr int BW = (TA + AL - 1 + AL - 1) / AL * AL;
+    static constexpr size_t box_elems = size_t(L::M) * TB * BW;
+    static constexpr size_t stage_elems = (box_elems * sizeof(Real) + 127) / 128 * 128 / sizeof(Real);
+    static constexpr size_t F_elems = size_t(Axes<L>::NMOVE) * NT;
+    static constexpr size_t bytes = (S * stage_elems + F_elems) * sizeof(Real) + S * sizeof(uint64_t) + 128;
+};
+
+template <int LAT, bool REC, typename Real, int TA, int TB, int S>
+__global__ void __launch_bounds__(TA *TB) mrlbm_step_kernel(const __grid_constant__ CUtensorMap tmap,
+                                                            const StepArgs p)
+{
+    using L = Lattice<LAT>;
+    using X = Axes<L>;
+    constexpr int D = L::D, Q = L::Q, M = L::M;
+    constexpr int HB = (D == 3) ? 1 : 0; // halo rows along B
+    constexpr int NT = TA * TB;
+    using SM = StepSmem<LAT, Real, TA, TB, S>;
+
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    Real *stage = reinterpret_cast<Real *>(smem_raw);
+    Real *Fs = stage + S * SM::stage_elems;
+    uint64_t *full = reinterpret_cast<uint64_t *>(Fs + SM::F_elems);
+
+    const int tid = threadIdx.x;
+    const int tx = tid % TA, ty = tid / TA;
+    const int tA = blockIdx.x % p.tilesA, tB = blockIdx.x / p.tilesA;
+    const int a0 = tA * (TA - 2) - 1;
+    const int b0 = (D == 3) ? tB * (TB - 2) - 1 : 0;
+    const int a = a0 + tx, b = b0 + ty;
+    const int nA = p.nA, nB = p.nB, nC = p.nC;
+
+    const int c0 = p.c_begin + blockIdx.y * p.seg_len;
+    const int c1 = min(c0 + p.seg_len, p.c_end);
+    if (c0 >= c1) return;
+    const int boxA = ((a0 + p.padA) / SM::AL) * SM::AL; // aligned TMA box origin (a0 + padA >= 0)
+    const int offA = a0 + p.padA - boxA;                  // window column 0 inside the box
+    const int cfirst = (c0 > 0 || p.lo_nb) ? c0 - 1 : c0;
+    const int clast = (c1 < nC || p.hi_nb) ? c1 : c1 - 1;
+    const int nl = clast - cfirst + 1;
+
+    // ---- per-thread roles
+    const bool perA = p.kind[0] == BC_PERIODIC, perB = p.kind[2] == BC_PERIODIC;
+    const bool inA = a >= 0 && a < nA, inB = b >= 0 && b < nB;
+    const bool valid = (inA || perA) && (inB || perB); // holds a real (possibly wrapped) node
+    const bool wrapped = valid && !(inA && inB);
+    const int aw = inA ? a : (a + nA) % nA;
+    const int bw = inB ? b : (b + nB) % nB;
+    const bool interior = tx >= 1 && tx < TA - 1 && ty >= HB && ty < TB - HB;
+    const bool owner = interior && inA && inB;
+    // pull-source availability along A/B: source at a-1 (c_a = +1), a+1 (c_a = -1)
+    const bool okAm = (a - 1 >= 0) || perA, okAp = (a + 1 < nA) || perA;
+    const bool okBm = (D == 2) || (b - 1 >= 0) || perB, okBp = (D == 2) || (b + 1 < nB) || perB;
+    // walls touching this node in-plane (-1 lower face, +1 upper face)
+    auto is_wall = [](int k) { return k == BC_WALL || k == BC_MOVING; };
+    const int bbA = (a == 0 && is_wall(p.kind[0])) ? -1 : ((a == nA - 1 && is_wall(p.kind[1])) ? 1 : 0);
+    const int bbB = (D == 2) ? 0 : ((b == 0 && is_wall(p.kind[2])) ? -1 : ((b == nB - 1 && is_wall(p.kind[3])) ? 1 : 0));
+    // open face of this node (index 0..3 into open_*), inward normal (physical x / y)
+    int openF = -1, nx_in = 0, ny_in = 0;
+    if (owner) {
+        if (a == 0 && p.kind[0] >= BC_VELOCITY) { openF = 0; nx_in = 1; }
+        else if (a == nA - 1 && p.kind[1] >= BC_VELOCITY) { openF = 1; nx_in = -1; }
+        else if (D == 3 && b == 0 && p.kind[2] >= BC_VELOCITY) { openF = 2; ny_in = 1; }
+        else if (D == 3 && b == nB - 1 && p.kind[3] >= BC_VELOCITY) { openF = 3; ny_in = -1; }
+    }
+
+    const Real *src = reinterpret_cast<const Real *>(p.src);
+    Real *dst = reinterpret_cast<Real *>(p.dst);
+    const Real omega = Real(p.omega);
+    auto plane_of = [&](int c) -> int { return p.wrapC ? ((c % nC + nC) % nC) + 1 : c + 1; };
+
+    // ---- TMA ring prologue
+    if (tid == 0) {
+        prefetch_tmap(&tmap);
+#pragma unroll
+        for (int s = 0; s < S; s++) mbar_init(&full[s], 1);
+        fence_barrier_init();
+    }
+    __syncthreads();
+    constexpr uint32_t stage_bytes = uint32_t(SM::box_elems * sizeof(Real)); // bytes one TMA box delivers
+    if (tid == 0) {
+        for (int s = 0; s < S && s < nl; s++) {
+            mbar_expect_tx(&full[s], stage_bytes);
+            tma_load_4d(stage + s * SM::stage_elems, &tmap, &full[s], boxA, b0 + p.padB, 0, plane_of(cfirst + s));
+        }
+    }
+
+    Real acc[3][M]; // rolling accumulators for layers c-1, c, c+1
+#pragma unroll
+    for (int j = 0; j < 3; j++)
+#pragma unroll
+        for (int q = 0; q < M; q++) acc[j][q] = Real(0);
+
+    // ---- finalize the completed layer and store it (eqs 1-3; open faces R14)
+    auto finalize_store = [&](const Real (&s)[M], int c) {
+        Real out[M];
+        const Real S0 = s[0];
+        if (openF < 0) {
+            const Real rho = Real(1) + S0;
+            const Real inv = Real(1) / rho;
+            out[0] = S0;
+#pragma unroll
+            for (int q = 0; q < D; q++) out[1 + q] = s[1 + q] * inv;
+#pragma unroll
+            for (int q = 0; q < D; q++)
+#pragma unroll
+                for (int r = q; r < D; r++)
+                    out[pslot<D>(q, r)] = s[pslot<D>(q, r)] - ((q == r) ? S0 * Real(1.0 / 3.0) : Real(0));
+        } else {
+            // weighted sums over K0 (x1) and K- (x2) populations:
+            //   S0 = sum wt f = S0~ + 1,  SPi = sum wt H f = acc - delta S0~/3
+            Real u[3] = {Real(0), Real(0), Real(0)};
+            Real drho;
+            const int kind = p.kind[openF];
+            if (kind == BC_VELOCITY) {
+                const double *prof = p.open_prof[openF];
+                if (prof) {
+                    const long long fi = (openF < 2) ? ((long long)(c + p.c_offset) * nB + b)
+                                                     : ((long long)(c + p.c_offset) * nA + a);
+#pragma unroll
+                    for (int q = 0; q < D; q++) u[q] = Real(prof[fi * D + q]);
+                } else {
+#pragma unroll
+                    for (int q = 0; q < D; q++) u[q] = Real(p.open_u[openF][q]);
+                }
+                const Real un = u[0] * Real(nx_in) + u[1] * Real(ny_in);
+                drho = (S0 + un) / (Real(1) - un);            // rho = S0 / (1 - u.n)
+            } else {
+                drho = Real(p.open_drho[openF]);
+                const Real rho = Real(1) + drho;
+                const Real un = (drho - S0) / rho;            // u.n = 1 - S0 / rho
+                u[0] = un * Real(nx_in);
+                u[1] = un * Real(ny_in);
+            }
+            const Real rho = Real(1) + drho;
+            out[0] = drho;
+#pragma unroll
+            for (int q = 0; q < D; q++) out[1 + q] = u[q];
+            // Pi = SPi - 2 sum_{K-} H f^eq,odd = SPi - 6 rho sum_{K-} w H (c.u)
+            Real corr[M];
+#pragma unroll
+            for (int q = 0; q < M; q++) corr[q] = Real(0);
+            static_for<0, Q>([&](auto kk) {
+                constexpr int k = decltype(kk)::value;
+                constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
+                constexpr Real wk = Real(L::w[k]);
+                const int cn = kx * nx_in + ky * ny_in;
+                if (cn < 0) {
+                    Real cu = Real(kx) * u[0] + Real(ky) * u[1];
+                    if constexpr (D == 3) cu += Real(kz) * u[2];
+                    const Real t = wk * cu;
+                    static_for<0, D>([&](auto qk) {
+                        constexpr int q = decltype(qk)::value;
+                        static_for<q, D>([&](auto rk) {
+                            constexpr int r = decltype(rk)::value;
+                            constexpr Real H = Real(L::c[k][q] * L::c[k][r]) - ((q == r) ? Real(1.0 / 3.0) : Real(0));
+                            corr[pslot<D>(q, r)] += H * t;
+                        });
+                    });
+                }
+            });
+#pragma unroll
+            for (int q = 0; q < D; q++)
+#pragma unroll
+                for (int r = q; r < D; r++)
+                    out[pslot<D>(q, r)] = s[pslot<D>(q, r)] - ((q == r) ? S0 * Real(1.0 / 3.0) : Real(0)) -
+                                          Real(6) * rho * corr[pslot<D>(q, r)];
+        }
+        Real *o = dst + (long long)(c + 1) * p.pstride + (long long)b * p.pitch + a;
+#pragma unroll
+        for (int q = 0; q < M; q++) o[q * p.mstride] = out[q];
+    };
+
+    for (int it = 0; it < nl; it++) {
+        const int c = cfirst + it;
+        const int s = it % S;
+        mbar_wait(&full[s], (it / S) & 1);
+
+        Real m[M];
+        if (valid) {
+            if (!wrapped) {
+                const Real *st = stage + s * SM::stage_elems + ty * SM::BW + tx + offA;
+#pragma unroll
+                for (int q = 0; q < M; q++) m[q] = st[q * (TB * SM::BW)];
+            } else {
+                const Real *g = src + (long long)plane_of(c) * p.pstride + (long long)bw * p.pitch + aw;
+#pragma unroll
+                for (int q = 0; q < M; q++) m[q] = g[q * p.mstride];
+            }
+        }
+        __syncthreads(); // stage s consumed; previous layer's F reads done
+        if (tid == 0 && it + S < nl) {
+            mbar_expect_tx(&full[s], stage_bytes);
+            tma_load_4d(stage + s * SM::stage_elems, &tmap, &full[s], boxA, b0 + p.padB, 0, plane_of(c + S));
+        }
+
+        // ---- collide + reconstruct (eqs 10-14) and publish in-plane movers
+        Real fown[Q]; // only the non-moving entries are used after the barrier
+        Real rho_own = Real(1);
+        if (valid) {
+            Real A[Basis<LAT, REC>::NH];
+            collide_coeffs<LAT, REC, Real>(m, omega, A);
+            reconstruct<LAT, REC, Real>(A, fown);
+            rho_own = Real(1) + m[0];
+            static_for<0, Q>([&](auto kk) {
+                constexpr int k = decltype(kk)::value;
+                if constexpr (X::moving(k)) Fs[X::slot(k) * NT + tid] = fown[k];
+            });
+        }
+        __syncthreads();
+
+        if (owner) {
+            const bool tgt_lo = (c > 0) || p.lo_nb;      // layer c-1 exists
+            const bool tgt_hi = (c < nC - 1) || p.hi_nb; // layer c+1 exists
+            const int bbC = (c == 0 && !p.lo_nb) ? -1 : ((c == nC - 1 && !p.hi_nb) ? 1 : 0);
+            auto body = [&](auto open_tag) {
+                constexpr bool OPEN = decltype(open_tag)::value;
+                auto wt = [&](int kx, int ky) -> Real {
+                    const int cn = kx * nx_in + ky * ny_in;
+                    return cn > 0 ? Real(0) : (cn < 0 ? Real(2) : Real(1));
+                };
+                // streaming (eq 7), pull form across the tile; C-moves in registers
+                static_for<0, Q>([&](auto kk) {
+                    constexpr int k = decltype(kk)::value;
+                    constexpr int ca = X::ca(k), cb = X::cb(k), cm = X::cm(k);
+                    const bool tgt = (cm == 0) || (cm < 0 ? tgt_lo : tgt_hi);
+                    bool ok = tgt;
+                    if constexpr (ca > 0) ok = ok && okAm;
+                    if constexpr (ca < 0) ok = ok && okAp;
+                    if constexpr (cb > 0) ok = ok && okBm;
+                    if constexpr (cb < 0) ok = ok && okBp;
+                    if (ok) {
+                        Real v;
+                        if constexpr (X::moving(k)) v = Fs[X::slot(k) * NT + (ty - cb) * TA + (tx - ca)];
+                        else v = fown[k];
+                        if constexpr (OPEN) {
+                            constexpr int kx = L::c[k][0], ky = L::c[k][1];
+                            v *= wt(kx, ky);
+                        }
+                        accum<L, k>(acc[cm + 1], v);
+                    }
+                });
+                // halfway bounce-back at walls (push form at the emitting node,
+                // R12) with the moving-wall term (R13)
+                if (bbA | bbB | bbC) {
+                    static_for<0, Q>([&](auto kk) {
+                        constexpr int k = decltype(kk)::value;
+                        constexpr int ca = X::ca(k), cb = X::cb(k), cm = X::cm(k);
+                        const bool xA = (ca != 0) && (ca == bbA);
+                        const bool xB = (cb != 0) && (cb == bbB);
+                        const bool xC = (cm != 0) && (cm == bbC);
+                        if (xA || xB || xC) {
+                            Real v;
+                            if constexpr (X::moving(k)) v = Fs[X::slot(k) * NT + tid];
+                            else v = fown[k];
+                            constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
+                            constexpr double wk6 = 6.0 * L::w[k];
+                            double cuw = 0.0;
+                            auto lid = [&](int face) {
+                                if (p.kind[face] == BC_MOVING)
+                                    cuw += kx * p.uw[face][0] + ky * p.uw[face][1] + kz * p.uw[face][2];
+                            };
+                            if (xA) lid(ca < 0 ? 0 : 1);
+                            if (xB) lid(cb < 0 ? 2 : 3);
+                            if (xC) lid(cm < 0 ? 4 : 5);
+                            v -= Real(wk6) * rho_own * Real(cuw);
+                            constexpr int ko = X::opp(k);
+                            if constexpr (OPEN) {
+                                constexpr int ox = L::c[ko][0], oy = L::c[ko][1];
+                                v *= wt(ox, oy);
+                            }
+                            accum<L, ko>(acc[1], v);
+                        }
+                    });
+                }
+            };
+            if (openF >= 0) body(std::true_type{});
+            else body(std::false_type{});
+
+            if (c - 1 >= c0 && c - 1 < c1) finalize_store(acc[0], c - 1);
+        }
+        // rotate the accumulator window
+#pragma unroll
+        for (int q = 0; q < M; q++) {
+            acc[0][q] = acc[1][q];
+            acc[1][q] = acc[2][q];
+            acc[2][q] = Real(0);
+        }
+    }
+    if (owner && clast == c1 - 1) finalize_store(acc[0], c1 - 1);
+}
+
+// ------------------------------------------------------------ side kernels
+struct GridArgs {
+    int nA, nB, nC, pitch;
+    long long mstride, pstride;
+};
+
+// ABI fp64 [M][nC][nB][nA] (rho, u, Pi) -> internal Real layout (rho - 1).
+template <int M, typename Real>
+__global__ void set_moments_kernel(const double *__restrict__ in, Real *__restrict__ buf, GridArgs g)
+{
+    const long long N = (long long)g.nA * g.nB * g.nC;
+    for (long long n = blockIdx.x * (long long)blockDim.x + threadIdx.x; n < N; n += (long long)gridDim.x * blockDim.x) {
+        const int a = n % g.nA;
+        const int b = (n / g.nA) % g.nB;
+        const int c = n / ((long long)g.nA * g.nB);
+        Real *o = buf + (long long)(c + 1) * g.pstride + (long long)b * g.pitch + a;
+#pragma unroll
+        for (int q = 0; q < M; q++) {
+            double v = in[q * N + n];
+            if (q == 0) v -= 1.0;
+            o[q * g.mstride] = Real(v);
+        }
+    }
+}
+
+template <int M, typename Real>
+__global__ void get_moments_kernel(const Real *__restrict__ buf, double *__restrict__ out, GridArgs g)
+{
+    const long long N = (long long)g.nA * g.nB * g.nC;
+    for (long long n = blockIdx.x * (long long)blockDim.x + threadIdx.x; n < N; n += (long long)gridDim.x * blockDim.x) {
+        const int a = n % g.nA;
+        const int b = (n / g.nA) % g.nB;
+        const int c = n / ((long long)g.nA * g.nB);
+        const Real *i = buf + (long long)(c + 1) * g.pstride + (long long)b * g.pitch + a;
+#pragma unroll
+        for (int q = 0; q < M; q++) {
+            double v = double(i[q * g.mstride]);
+            if (q == 0) v += 1.0;
+            out[q * N + n] = v;
+        }
+    }
+}
+
+// Post-collision populations f* = f~* + w of every node (R17), fp64 [Q][N].
+template <int LAT, bool REC, typename Real>
+__global__ void populations_kernel(const Real *__restrict__ buf, double *__restrict__ out, GridArgs g, double omega)
+{
+    using L = Lattice<LAT>;
+    const long long N = (long long)g.nA * g.nB * g.nC;
+    for (long long n = blockIdx.x * (long long)blockDim.x + threadIdx.x; n < N; n += (long long)gridDim.x * blockDim.x) {
+        const int a = n % g.nA;
+        const int b = (n / g.nA) % g.nB;
+        const int c = n / ((long long)g.nA * g.nB);
+        const Real *i = buf + (long long)(c + 1) * g.pstride + (long long)b * g.pitch + a;
+        Real m[L::M];
+#pragma unroll
+        for (int q = 0; q < L::M; q++) m[q] = i[q * g.mstride];
+        Real A[Basis<LAT, REC>::NH];
+        Real f[L::Q];
+        collide_coeffs<LAT, REC, Real>(m, Real(omega), A);
+        reconstruct<LAT, REC, Real>(A, f);
+        static_for<0, L::Q>([&](auto kk) {
+            constexpr int k = decltype(kk)::value;
+            constexpr double wk = L::w[k];
+            out[k * N + n] = double(f[k]) + wk;
+        });
+    }
+}
+
+template <int M, typename Real>
+__global__ void finite_kernel(const Real *__restrict__ buf, GridArgs g, int *flag)
+{
+    const long long N = (long long)g.nA * g.nB * g.nC;
+    for (long long n = blockIdx.x * (long long)blockDim.x + threadIdx.x; n < N; n += (long long)gridDim.x * blockDim.x) {
+        const int a = n % g.nA;
+        const int b = (n / g.nA) % g.nB;
+        const int c = n / ((long long)g.nA * g.nB);
+        const Real *i = buf + (long long)(c + 1) * g.pstride + (long long)b * g.pitch + a;
+#pragma unroll
+        for (int q = 0; q < M; q++)
+            if (!isfinite(double(i[q * g.mstride]))) atomicExch(flag, 1);
+    }
+}
+
+} // namespace mr

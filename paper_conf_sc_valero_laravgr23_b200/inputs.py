@@ -72,6 +72,22 @@ def perturbed_rest(D, nx, ny, nz=1, U=0.05, seed=SEED, pi_neq=True):
     return pack(rho, u, Pi)
 
 
+def smooth_state(D, nx, ny, nz=1, U=0.05, seed=SEED):
+    """Smooth seeded flow of order U: 4 random-phase modes on every moment
+    (rho: 1e-2, u: U, Pi^neq: 1e-3 U) -- parity tests (every Hermite term
+    and every velocity component is O(U), so the per-group metric is not
+    dominated by absolute rounding of near-zero fields)."""
+    rng = np.random.default_rng(seed)
+    g = _grid(D, nx, ny, nz)
+    rho = 1.0 + _modes(rng, g, 1e-2)
+    u = [_modes(rng, g, U) for _ in range(D)]
+    Pi = [[None] * D for _ in range(D)]
+    for a in range(D):
+        for b in range(a, D):
+            Pi[a][b] = Pi[b][a] = rho * u[a] * u[b] + _modes(rng, g, 1e-3 * U)
+    return pack(rho, u, Pi)
+
+
 def random_state(D, nx, ny, nz=1, U=0.05, seed=SEED):
     """Non-smooth seeded state: i.i.d. noise on every moment (parity stress test)."""
     rng = np.random.default_rng(seed)
