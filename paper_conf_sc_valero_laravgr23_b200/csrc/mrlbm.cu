@@ -60,7 +60,7 @@ struct Variant {
 
 inline int grid_for(long long n) { return (int)std::min<long long>((n + 255) / 256, 148LL * 16); }
 
-template <int LAT, bool REC, typename Real, int TA, int TB, int S> Variant make_variant()
+template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB> Variant make_variant()
 {
     using L = mr::Lattice<LAT>;
     using SM = mr::StepSmem<LAT, Real, TA, TB, S>;
@@ -70,9 +70,9 @@ template <int LAT, bool REC, typename Real, int TA, int TB, int S> Variant make_
     v.S = S;
     v.BW = SM::BW;
     v.smem = SM::bytes;
-    v.kernel_fn = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S>;
+    v.kernel_fn = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB>;
     v.step = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
-        mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S><<<grid, TA * TB, SM::bytes, st>>>(map, a);
+        mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB><<<grid, TA * TB, SM::bytes, st>>>(map, a);
     };
     v.set = [](const double *in, void *buf, mr::GridArgs g, cudaStream_t st) {
         mr::set_moments_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
@@ -97,8 +97,8 @@ template <int LAT, bool REC, typename Real, int TA, int TB, int S> Variant make_
 // nodes); 3D 32 x 8 threads (30 x 6 interior nodes) with a 3-deep TMA ring.
 template <int LAT, bool REC, typename Real> Variant pick()
 {
-    if constexpr (LAT == mr::LAT_D2Q9) return make_variant<LAT, REC, Real, 128, 1, 4>();
-    else return make_variant<LAT, REC, Real, 32, 8, 3>();
+    if constexpr (LAT == mr::LAT_D2Q9) return make_variant<LAT, REC, Real, 128, 1, 4, 5>();
+    else return make_variant<LAT, REC, Real, 32, 8, 3, 2>();
 }
 
 Variant select_variant(int lat, int reg, int prec)
@@ -447,7 +447,9 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
 
     h->var = select_variant(lattice, reg, o.precision);
     if (cudaFuncSetAttribute(h->var.kernel_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)h->var.smem) !=
-        cudaSuccess)
+            cudaSuccess ||
+        cudaFuncSetAttribute(h->var.kernel_fn, cudaFuncAttributePreferredSharedMemoryCarveout,
+                             (int)cudaSharedmemCarveoutMaxShared) != cudaSuccess)
         return cleanup_fail(fail(MRLBM_ERR_CUDA, "smem attribute"));
 
     // TMA descriptors: tensor {nA, nB, M, nC + 2} of the [plane][m][b][a] layout

@@ -103,8 +103,10 @@ __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map)
 // closed form of Malaspinas' recursion, R8):
 //   n = 0: rho - 1 (shifted zeroth moment)     n = 1: rho u_a
 //   n = 2: omega Pi_ab + (1 - omega) rho u_a u_b           (= Pi*, eq 10)
-//   n > 2: rho prod u + omega sum_{p<q} Pneq_{a_p a_q} prod_{k != p,q} u_{a_k}
-// each times hscale(h).
+//   n > 2: rho u^h + omega sum_{pairs p<q} Pneq_{a_p a_q} u^{h - e_{a_p} - e_{a_q}}
+// each times hscale(h).  The pair sum is grouped by pair type: (a,a) occurs
+// C(h_a, 2) times and (a,b), a < b, h_a h_b times, so every term is one FMA
+// against a monomial u^m (m <= (2,2,2)) computed once per node.
 template <int LAT, bool REC, typename Real>
 __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M], Real omega,
                                                Real (&A)[Basis<LAT, REC>::NH])
@@ -120,6 +122,7 @@ __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M],
     u[2] = (D == 3) ? m[3] : Real(0);
     const Real omc = Real(1) - omega;
     Real Pn[3][3]; // Pi^neq (eq 8 in moment form: Pi - rho u u)
+    Real up[3][3]; // up[a][k] = u_a^k
     if constexpr (REC) {
 #pragma unroll
         for (int a = 0; a < D; a++)
@@ -128,13 +131,31 @@ __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M],
                 Pn[a][b] = m[pslot<D>(a, b)] - rho * u[a] * u[b];
                 Pn[b][a] = Pn[a][b];
             }
+#pragma unroll
+        for (int a = 0; a < 3; a++) {
+            up[a][0] = Real(1);
+            up[a][1] = u[a];
+            up[a][2] = u[a] * u[a];
+        }
     }
+    // u^(m0,m1,m2); factors equal to 1 are dropped at compile time
+    auto mono = [&](auto m0c, auto m1c, auto m2c) -> Real {
+        constexpr int m0 = decltype(m0c)::value, m1 = decltype(m1c)::value, m2 = decltype(m2c)::value;
+        if constexpr (m0 + m1 + m2 == 0) return Real(1);
+        else if constexpr (m1 + m2 == 0) return up[0][m0];
+        else if constexpr (m0 + m2 == 0) return up[1][m1];
+        else if constexpr (m0 + m1 == 0) return up[2][m2];
+        else if constexpr (m2 == 0) return up[0][m0] * up[1][m1];
+        else if constexpr (m1 == 0) return up[0][m0] * up[2][m2];
+        else if constexpr (m0 == 0) return up[1][m1] * up[2][m2];
+        else return up[0][m0] * up[1][m1] * up[2][m2];
+    };
+    using I0 = std::integral_constant<int, 0>;
     static_for<0, B::NH>([&](auto hk) {
         constexpr int k = decltype(hk)::value;
         constexpr int h0 = B::h[k][0], h1 = B::h[k][1], h2 = B::h[k][2];
         constexpr int n = h0 + h1 + h2;
         constexpr Real sc = Real(hscale(h0, h1, h2));
-        // axis labels of the component
         constexpr int i0 = (h0 > 0) ? 0 : ((h1 > 0) ? 1 : 2);
         Real val;
         if constexpr (n == 0) {
@@ -145,27 +166,85 @@ __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M],
             constexpr int i1 = (h0 == 2) ? 0 : ((h0 == 1) ? ((h1 > 0) ? 1 : 2) : ((h1 == 2) ? 1 : 2));
             val = omega * m[pslot<D>(i0, i1)] + omc * rho * u[i0] * u[i1];
         } else {
-            constexpr int idx[6] = {
-                0 < h0 ? 0 : (0 < h0 + h1 ? 1 : 2), 1 < h0 ? 0 : (1 < h0 + h1 ? 1 : 2),
-                2 < h0 ? 0 : (2 < h0 + h1 ? 1 : 2), 3 < h0 ? 0 : (3 < h0 + h1 ? 1 : 2),
-                4 < h0 ? 0 : (4 < h0 + h1 ? 1 : 2), 5 < h0 ? 0 : (5 < h0 + h1 ? 1 : 2)};
-            Real aeq = rho;
-#pragma unroll
-            for (int t = 0; t < n; t++) aeq *= u[idx[t]];
+            using H0 = std::integral_constant<int, h0>;
+            using H1 = std::integral_constant<int, h1>;
+            using H2 = std::integral_constant<int, h2>;
             Real aneq = Real(0);
-#pragma unroll
-            for (int p = 0; p < n; p++)
-#pragma unroll
-                for (int q = p + 1; q < n; q++) {
-                    Real t = Pn[idx[p]][idx[q]];
-#pragma unroll
-                    for (int r = 0; r < n; r++)
-                        if (r != p && r != q) t *= u[idx[r]];
-                    aneq += t;
-                }
-            val = aeq + omega * aneq;
+            // (a,a) pairs: C(h_a, 2) = 1 iff h_a == 2
+            if constexpr (h0 == 2) aneq = fma(Pn[0][0], mono(I0{}, H1{}, H2{}), aneq);
+            if constexpr (h1 == 2) aneq = fma(Pn[1][1], mono(H0{}, I0{}, H2{}), aneq);
+            if constexpr (h2 == 2) aneq = fma(Pn[2][2], mono(H0{}, H1{}, I0{}), aneq);
+            // (a,b) pairs: h_a h_b of them
+            if constexpr (h0 * h1 > 0)
+                aneq = fma(Real(h0 * h1) * Pn[0][1],
+                           mono(std::integral_constant<int, h0 - 1>{}, std::integral_constant<int, h1 - 1>{}, H2{}), aneq);
+            if constexpr (h0 * h2 > 0)
+                aneq = fma(Real(h0 * h2) * Pn[0][2],
+                           mono(std::integral_constant<int, h0 - 1>{}, H1{}, std::integral_constant<int, h2 - 1>{}), aneq);
+            if constexpr (h1 * h2 > 0)
+                aneq = fma(Real(h1 * h2) * Pn[1][2],
+                           mono(H0{}, std::integral_constant<int, h1 - 1>{}, std::integral_constant<int, h2 - 1>{}), aneq);
+            val = fma(omega, aneq, rho * mono(H0{}, H1{}, H2{}));
         }
         A[k] = val * sc;
+    });
+}
+
+template <int LAT, bool REC> constexpr int hindex(int a, int b, int c)
+{
+    for (int k = 0; k < Basis<LAT, REC>::NH; k++)
+        if (Basis<LAT, REC>::h[k][0] == a && Basis<LAT, REC>::h[k][1] == b && Basis<LAT, REC>::h[k][2] == c) return k;
+    return -1;
+}
+
+// 1D scaled Hermite synthesis at c = -1, 0, +1:
+//   g(c) = A0 + c A1 + (3c^2 - 1) A2  ->  g(0) = A0 - A2,  g(+-1) = A0 + 2 A2 +- A1
+template <typename Real>
+__device__ __forceinline__ void synth3(Real A0, Real A1, Real A2, Real &gm, Real &g0, Real &gp)
+{
+    const Real S = fma(Real(2), A2, A0);
+    g0 = A0 - A2;
+    gp = S + A1;
+    gm = S - A1;
+}
+
+// Sum-factorised eq 14 for the full tensor bases {0,1,2}^D (D2Q9 / D3Q27
+// recursive): the Hermite-to-population map is the D-fold tensor product of
+// the 1D map above, applied axis by axis (z, y, x), then times w_i.
+template <int LAT, typename Real>
+__device__ __forceinline__ void reconstruct_tensor(const Real (&A)[Basis<LAT, true>::NH], Real (&f)[Lattice<LAT>::Q])
+{
+    using L = Lattice<LAT>;
+    constexpr int D = L::D;
+    Real T[3][3][3]; // [h_x][h_y][c_z + 1]
+    static_for<0, 9>([&](auto abk) {
+        constexpr int a = decltype(abk)::value / 3, b = decltype(abk)::value % 3;
+        constexpr int k0 = hindex<LAT, true>(a, b, 0);
+        static_assert(k0 >= 0, "basis component missing");
+        if constexpr (D == 3) {
+            constexpr int k1 = hindex<LAT, true>(a, b, 1), k2 = hindex<LAT, true>(a, b, 2);
+            static_assert(k1 >= 0 && k2 >= 0, "basis component missing");
+            synth3(A[k0], A[k1], A[k2], T[a][b][0], T[a][b][1], T[a][b][2]);
+        } else {
+            T[a][b][1] = A[k0];
+        }
+    });
+    constexpr int z0 = (D == 3) ? 0 : 1, z1 = (D == 3) ? 3 : 2;
+    Real U[3][3][3]; // [h_x][c_y + 1][c_z + 1]
+#pragma unroll
+    for (int a = 0; a < 3; a++)
+#pragma unroll
+        for (int zi = z0; zi < z1; zi++) synth3(T[a][0][zi], T[a][1][zi], T[a][2][zi], U[a][0][zi], U[a][1][zi], U[a][2][zi]);
+    Real V[3][3][3]; // [c_x + 1][c_y + 1][c_z + 1]
+#pragma unroll
+    for (int yi = 0; yi < 3; yi++)
+#pragma unroll
+        for (int zi = z0; zi < z1; zi++) synth3(U[0][yi][zi], U[1][yi][zi], U[2][yi][zi], V[0][yi][zi], V[1][yi][zi], V[2][yi][zi]);
+    static_for<0, L::Q>([&](auto ik) {
+        constexpr int i = decltype(ik)::value;
+        constexpr Real w = Real(L::w[i]);
+        constexpr int xi = L::c[i][0] + 1, yi = L::c[i][1] + 1, zi = L::c[i][2] + 1;
+        f[i] = w * V[xi][yi][zi];
     });
 }
 
@@ -185,6 +264,10 @@ __device__ __forceinline__ void reconstruct(const Real (&A)[Basis<LAT, REC>::NH]
 {
     using L = Lattice<LAT>;
     using B = Basis<LAT, REC>;
+    if constexpr (REC && LAT != LAT_D3Q19) {
+        reconstruct_tensor<LAT, Real>(A, f);
+        return;
+    }
     static_for<0, L::HALF + 1>([&](auto ik) {
         constexpr int i = decltype(ik)::value;
         Real E = Real(0), O = Real(0);
@@ -236,8 +319,8 @@ template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
     static constexpr size_t bytes = (S * stage_elems + F_elems) * sizeof(Real) + S * sizeof(uint64_t) + 128;
 };
 
-template <int LAT, bool REC, typename Real, int TA, int TB, int S>
-__global__ void __launch_bounds__(TA *TB) mrlbm_step_kernel(const __grid_constant__ CUtensorMap tmap,
+template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB>
+__global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_constant__ CUtensorMap tmap,
                                                             const StepArgs p)
 {
     using L = Lattice<LAT>;
@@ -449,27 +532,38 @@ __global__ void __launch_bounds__(TA *TB) mrlbm_step_kernel(const __grid_constan
                     const int cn = kx * nx_in + ky * ny_in;
                     return cn > 0 ? Real(0) : (cn < 0 ? Real(2) : Real(1));
                 };
-                // streaming (eq 7), pull form across the tile; C-moves in registers
-                static_for<0, Q>([&](auto kk) {
-                    constexpr int k = decltype(kk)::value;
-                    constexpr int ca = X::ca(k), cb = X::cb(k), cm = X::cm(k);
-                    const bool tgt = (cm == 0) || (cm < 0 ? tgt_lo : tgt_hi);
-                    bool ok = tgt;
-                    if constexpr (ca > 0) ok = ok && okAm;
-                    if constexpr (ca < 0) ok = ok && okAp;
-                    if constexpr (cb > 0) ok = ok && okBm;
-                    if constexpr (cb < 0) ok = ok && okBp;
-                    if (ok) {
-                        Real v;
-                        if constexpr (X::moving(k)) v = Fs[X::slot(k) * NT + (ty - cb) * TA + (tx - ca)];
-                        else v = fown[k];
-                        if constexpr (OPEN) {
-                            constexpr int kx = L::c[k][0], ky = L::c[k][1];
-                            v *= wt(kx, ky);
+                // streaming (eq 7), pull form across the tile; C-moves stay in
+                // registers.  Arrivals for layer c-1 first, so that layer c-1
+                // is finalized and its accumulators freed before layers c, c+1
+                // are accumulated (lower register pressure).
+                auto pull = [&](auto cm_tag) {
+                    constexpr int CM = decltype(cm_tag)::value;
+                    static_for<0, Q>([&](auto kk) {
+                        constexpr int k = decltype(kk)::value;
+                        constexpr int ca = X::ca(k), cb = X::cb(k), cm = X::cm(k);
+                        if constexpr (cm == CM) {
+                            bool ok = (cm == 0) || (cm < 0 ? tgt_lo : tgt_hi);
+                            if constexpr (ca > 0) ok = ok && okAm;
+                            if constexpr (ca < 0) ok = ok && okAp;
+                            if constexpr (cb > 0) ok = ok && okBm;
+                            if constexpr (cb < 0) ok = ok && okBp;
+                            if (ok) {
+                                Real v;
+                                if constexpr (X::moving(k)) v = Fs[X::slot(k) * NT + (ty - cb) * TA + (tx - ca)];
+                                else v = fown[k];
+                                if constexpr (OPEN) {
+                                    constexpr int kx = L::c[k][0], ky = L::c[k][1];
+                                    v *= wt(kx, ky);
+                                }
+                                accum<L, k>(acc[cm + 1], v);
+                            }
                         }
-                        accum<L, k>(acc[cm + 1], v);
-                    }
-                });
+                    });
+                };
+                pull(std::integral_constant<int, -1>{});
+                if (c - 1 >= c0 && c - 1 < c1) finalize_store(acc[0], c - 1);
+                pull(std::integral_constant<int, 0>{});
+                pull(std::integral_constant<int, 1>{});
                 // halfway bounce-back at walls (push form at the emitting node,
                 // R12) with the moving-wall term (R13)
                 if (bbA | bbB | bbC) {
@@ -506,8 +600,6 @@ __global__ void __launch_bounds__(TA *TB) mrlbm_step_kernel(const __grid_constan
             };
             if (openF >= 0) body(std::true_type{});
             else body(std::false_type{});
-
-            if (c - 1 >= c0 && c - 1 < c1) finalize_store(acc[0], c - 1);
         }
         // rotate the accumulator window
 #pragma unroll
