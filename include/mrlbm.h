@@ -84,7 +84,8 @@ typedef struct {
     int device;                /* CUDA device ordinal, default current (-1) */
     void *cuda_stream;         /* cudaStream_t to enqueue on; NULL = own stream */
     int rank, nranks;          /* z-slab decomposition (2D: y-slabs); default 0, 1 */
-    const void *nccl_unique_id;/* 128-byte ncclUniqueId, required if nranks > 1 */
+    const void *nccl_unique_id;/* 128-byte ncclUniqueId for nranks > 1 (one GPU per
+                                  rank); NULL with nranks > 1 = slab-group mode */
 } mrlbm_options;
 
 typedef int mrlbm_status;
@@ -155,6 +156,26 @@ const char *mrlbm_last_error(void); /* thread-local detail of the last error */
 /* Write a 128-byte ncclUniqueId into id (rank 0 creates it, then it is
  * broadcast out of band, e.g. through torch.distributed). */
 mrlbm_status mrlbm_nccl_unique_id(void *id128);
+
+/* Slab-group mode (one process, one device): handles created with nranks = P,
+ * rank = r and nccl_unique_id = NULL form one z-slab decomposition whose halo
+ * planes are exchanged with device-to-device copies instead of NCCL.  Advance
+ * all P slabs by n steps (enqueued on handles[0]'s stream; each handle's own
+ * stream is ordered before and after).  mrlbm_step on such a handle returns
+ * MRLBM_ERR_INVALID_ARGUMENT.  Used to verify the decomposition on one GPU. */
+mrlbm_status mrlbm_step_group(mrlbm_t *handles, int n_handles, int64_t n);
+
+/* Host-only helpers (no CUDA calls): the slab partition of an extent n over
+ * nranks (remainder to the first ranks), and the argument validation that
+ * mrlbm_create performs (returns the status mrlbm_create would return). */
+mrlbm_status mrlbm_partition(int64_t n, int nranks, int rank, int64_t *n_local, int64_t *offset);
+mrlbm_status mrlbm_validate(mrlbm_lattice lattice, int64_t nx, int64_t ny, int64_t nz, double tau,
+                            mrlbm_regularization reg, const mrlbm_boundary *boundary, int nranks);
+
+/* Fused-kernel launch configuration of a handle (tile TA x TB threads, TMA
+ * stages S, sweep segment length, grid, dynamic shared memory bytes). */
+mrlbm_status mrlbm_kernel_config(mrlbm_t h, int *TA, int *TB, int *S, int *seg_len, int *grid_x, int *grid_y,
+                                 int64_t *smem_bytes);
 
 #ifdef __cplusplus
 }

@@ -94,24 +94,37 @@ template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB> Var
 }
 
 // Tile shapes: 2D one row of 128 threads (126 interior
-// nodes); 3D 32 x 8 threads (30 x 6 interior nodes) with a 3-deep TMA ring.
-template <int LAT, bool REC, typename Real> Variant pick()
+// nodes); 3D either 32 x 8 threads (30 x 6 interior, 2 CTAs/SM) or 32 x 16
+// threads (30 x 14 interior, 1 CTA/SM).  tile = 0: library default, 1: 32x8,
+// 2: 32x16 (MRLBM_TILE overrides, for tuning).
+template <int LAT, bool REC, typename Real> Variant pick(int tile)
 {
-    if constexpr (LAT == mr::LAT_D2Q9) return make_variant<LAT, REC, Real, 128, 1, 4, 5>();
-    else return make_variant<LAT, REC, Real, 32, 8, 3, 2>();
+    if constexpr (LAT == mr::LAT_D2Q9) {
+        return make_variant<LAT, REC, Real, 128, 1, 4, 5>();
+    } else {
+        constexpr bool big = LAT == mr::LAT_D3Q27 && sizeof(Real) == 8; // 24 movers x 512 x 8 B
+        if (tile == 1) return make_variant<LAT, REC, Real, 32, 8, 3, 2>();
+        return make_variant<LAT, REC, Real, 32, 16, (big ? 2 : 3), 1>();
+    }
 }
 
-Variant select_variant(int lat, int reg, int prec)
+Variant select_variant(int lat, int reg, int prec, int tile)
 {
     const bool R = reg == MRLBM_RECURSIVE;
     const bool F = prec == MRLBM_FP32;
 #define MR_SEL(LAT)                                                                                 \
-    if (R) return F ? pick<LAT, true, float>() : pick<LAT, true, double>();                         \
-    else return F ? pick<LAT, false, float>() : pick<LAT, false, double>();
+    if (R) return F ? pick<LAT, true, float>(tile) : pick<LAT, true, double>(tile);                 \
+    else return F ? pick<LAT, false, float>(tile) : pick<LAT, false, double>(tile);
     if (lat == MRLBM_D2Q9) { MR_SEL(mr::LAT_D2Q9) }
     if (lat == MRLBM_D3Q19) { MR_SEL(mr::LAT_D3Q19) }
     MR_SEL(mr::LAT_D3Q27)
 #undef MR_SEL
+}
+
+int env_int(const char *name, int dflt)
+{
+    const char *v = getenv(name);
+    return v && *v ? atoi(v) : dflt;
 }
 
 typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
@@ -159,6 +172,7 @@ struct mrlbm_ctx {
     size_t io_bytes = 0;
     int *flag = nullptr;
     ncclComm_t comm = nullptr;
+    bool group_mode = false;    // nranks > 1 without NCCL: ghosts filled by mrlbm_step_group
     int nb_lo = -1, nb_hi = -1; // neighbour ranks along C (-1 none)
     cudaGraphExec_t graph[2] = {nullptr, nullptr};
     int graph_steps = 0;
@@ -179,6 +193,8 @@ mr::GridArgs grid_args(const mrlbm_ctx *h)
     g.pitch = h->pitch;
     g.mstride = h->mstride;
     g.pstride = h->pstride;
+    g.perA = h->base.kind[0] == mr::BC_PERIODIC;
+    g.perB = h->D == 3 && h->base.kind[2] == mr::BC_PERIODIC;
     return g;
 }
 
@@ -355,7 +371,6 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     if (o.precision != MRLBM_FP64 && o.precision != MRLBM_FP32) return fail(MRLBM_ERR_INVALID_ARGUMENT, "precision");
     mrlbm_status st = mrlbm_validate(lattice, nx, ny, nz, tau, reg, boundary, o.nranks);
     if (st) return st;
-    if (o.nranks > 1 && !o.nccl_unique_id) return fail(MRLBM_ERR_INVALID_ARGUMENT, "nranks > 1 needs nccl_unique_id");
     if (o.rank < 0 || o.rank >= o.nranks) return fail(MRLBM_ERR_INVALID_ARGUMENT, "rank out of range");
 
     EncodeTiledFn encode = get_encode_fn();
@@ -397,8 +412,10 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     h->padA = 16 / h->wbytes;
     h->padB = h->D == 3 ? 1 : 0;
     const int align = 32 / h->wbytes;
-    h->pitch = (h->padA + h->nA + align - 1) / align * align;
-    h->mstride = (long long)(h->padB + h->nB) * h->pitch;
+    // one extra column (and, in 3D, row) after the last node: the high-side
+    // periodic ghosts (the low-side ghosts live in the pads)
+    h->pitch = (h->padA + h->nA + 1 + align - 1) / align * align;
+    h->mstride = (long long)(h->padB + h->nB + h->padB) * h->pitch;
     h->origin = (long long)h->padB * h->pitch + h->padA;
     h->pstride = (long long)h->M * h->mstride;
     h->buf_bytes = (size_t)(h->nC + 2) * h->pstride * h->wbytes;
@@ -445,7 +462,7 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
         f.u_profile = nullptr;
     }
 
-    h->var = select_variant(lattice, reg, o.precision);
+    h->var = select_variant(lattice, reg, o.precision, env_int("MRLBM_TILE", 0));
     if (cudaFuncSetAttribute(h->var.kernel_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)h->var.smem) !=
             cudaSuccess ||
         cudaFuncSetAttribute(h->var.kernel_fn, cudaFuncAttributePreferredSharedMemoryCarveout,
@@ -454,8 +471,8 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
 
     // TMA descriptors: tensor {nA, nB, M, nC + 2} of the [plane][m][b][a] layout
     for (int i = 0; i < 2; i++) {
-        cuuint64_t dims[4] = {(cuuint64_t)(h->padA + h->nA), (cuuint64_t)(h->padB + h->nB), (cuuint64_t)h->M,
-                              (cuuint64_t)(h->nC + 2)};
+        cuuint64_t dims[4] = {(cuuint64_t)(h->padA + h->nA + 1), (cuuint64_t)(h->padB + h->nB + h->padB),
+                              (cuuint64_t)h->M, (cuuint64_t)(h->nC + 2)};
         cuuint64_t strides[3] = {(cuuint64_t)h->pitch * h->wbytes, (cuuint64_t)h->mstride * h->wbytes,
                                  (cuuint64_t)h->pstride * h->wbytes};
         cuuint32_t box[4] = {(cuuint32_t)h->var.BW, (cuuint32_t)h->var.TB, (cuuint32_t)h->M, 1};
@@ -512,18 +529,27 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     h->tilesA = (h->nA + TA - 3) / (TA - 2);
     h->tilesB = h->D == 3 ? (h->nB + TB - 3) / (TB - 2) : 1;
     a.tilesA = h->tilesA;
-    // segments along C: aim for >= 8 resident waves of CTAs, segments >= 8 layers
+    // segments along C: short enough that the resident CTAs sweep nearby
+    // layers together (their halo re-reads then hit L2) and that there are
+    // >= ~4 waves of CTAs; >= 8 layers so the two halo layers per segment
+    // stay cheap.  MRLBM_SEG overrides (tuning).
     {
         const long long tiles = (long long)h->tilesA * h->tilesB;
-        const long long target = 148LL * 8;
-        long long nseg = std::max<long long>(1, target / std::max<long long>(1, tiles));
-        long long seg = (h->nC + nseg - 1) / nseg;
+        long long seg = env_int("MRLBM_SEG", 0);
+        if (seg <= 0) {
+            const long long target = 148LL * 4 * 4;
+            const long long nseg = std::max<long long>(1, target / std::max<long long>(1, tiles));
+            seg = (h->nC + nseg - 1) / nseg;
+            seg = std::min<long long>(seg, 64);
+        }
         seg = std::max<long long>(seg, std::min<long long>(8, h->nC));
+        seg = std::min<long long>(seg, h->nC);
         h->seg_len = (int)seg;
         h->nseg = (int)((h->nC + seg - 1) / seg);
     }
 
-    if (h->nranks > 1) {
+    h->group_mode = h->nranks > 1 && !o.nccl_unique_id;
+    if (h->nranks > 1 && !h->group_mode) {
         if (cudaStreamCreateWithFlags(&h->comm_stream, cudaStreamNonBlocking) != cudaSuccess)
             return cleanup_fail(fail(MRLBM_ERR_CUDA, "comm stream"));
         ncclUniqueId id;
@@ -625,6 +651,7 @@ static const int kGraphSteps = 32; // even: a replay returns the ping-pong parit
 mrlbm_status mrlbm_step(mrlbm_t h, int64_t n)
 {
     if (!h || n < 0) return fail(MRLBM_ERR_INVALID_ARGUMENT, "bad step count");
+    if (h->group_mode) return fail(MRLBM_ERR_INVALID_ARGUMENT, "slab-group handle: use mrlbm_step_group");
     // Batches of kGraphSteps single-rank steps are replayed from a captured graph.
     while (h->nranks == 1 && n >= kGraphSteps) {
         const int par = h->cur;
@@ -705,6 +732,53 @@ mrlbm_status mrlbm_time_steps(mrlbm_t h, int64_t n, double *ms_per_step)
     float ms = 0.f;
     MR_CUDA(cudaEventElapsedTime(&ms, h->ev_t0, h->ev_t1));
     *ms_per_step = ms / (double)n;
+    return MRLBM_OK;
+}
+
+// Single-process slab group: handles[r] is rank r of one decomposition created
+// with nranks = n_handles and no NCCL id, all on the same device.  Per step the
+// boundary planes move into the neighbours' ghost planes with device-to-device
+// copies (the transport NCCL provides across GPUs), then every slab runs the
+// same interior / boundary launches as the NCCL path.  All work is ordered on
+// handles[0]'s stream.
+mrlbm_status mrlbm_step_group(mrlbm_t *hs, int n_handles, int64_t n)
+{
+    if (!hs || n_handles < 2 || n < 0) return fail(MRLBM_ERR_INVALID_ARGUMENT, "bad group");
+    for (int r = 0; r < n_handles; r++)
+        if (!hs[r] || !hs[r]->group_mode || hs[r]->rank != r || hs[r]->nranks != n_handles ||
+            hs[r]->device != hs[0]->device || hs[r]->prec != hs[0]->prec || hs[r]->pstride != hs[0]->pstride)
+            return fail(MRLBM_ERR_INVALID_ARGUMENT, "handles are not ranks 0..P-1 of one slab group");
+    cudaStream_t st = hs[0]->stream;
+    for (int r = 1; r < n_handles; r++) {
+        MR_CUDA(cudaEventRecord(hs[r]->ev_ready, hs[r]->stream));
+        MR_CUDA(cudaStreamWaitEvent(st, hs[r]->ev_ready, 0));
+    }
+    for (int64_t t = 0; t < n; t++) {
+        for (int r = 0; r < n_handles; r++) {
+            mrlbm_ctx *h = hs[r];
+            const size_t plane = (size_t)h->pstride * h->wbytes;
+            char *mine = (char *)h->buf[h->cur];
+            if (h->nb_lo >= 0) {
+                mrlbm_ctx *g = hs[h->nb_lo];
+                MR_CUDA(cudaMemcpyAsync(mine, (char *)g->buf[g->cur] + plane * g->nC, plane, cudaMemcpyDeviceToDevice, st));
+            }
+            if (h->nb_hi >= 0) {
+                mrlbm_ctx *g = hs[h->nb_hi];
+                MR_CUDA(cudaMemcpyAsync(mine + plane * (h->nC + 1), (char *)g->buf[g->cur] + plane * 1, plane,
+                                        cudaMemcpyDeviceToDevice, st));
+            }
+        }
+        for (int r = 0; r < n_handles; r++) {
+            mrlbm_ctx *h = hs[r];
+            launch_range(h, h->cur, 1, h->nC - 1, st);
+            launch_range(h, h->cur, 0, 1, st);
+            launch_range(h, h->cur, h->nC - 1, h->nC, st);
+        }
+        for (int r = 0; r < n_handles; r++) hs[r]->cur ^= 1;
+        MR_CUDA(cudaGetLastError());
+    }
+    MR_CUDA(cudaEventRecord(hs[0]->ev_ready, st));
+    for (int r = 1; r < n_handles; r++) MR_CUDA(cudaStreamWaitEvent(hs[r]->stream, hs[0]->ev_ready, 0));
     return MRLBM_OK;
 }
 

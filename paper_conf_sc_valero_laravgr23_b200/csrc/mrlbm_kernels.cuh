@@ -355,12 +355,15 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     // ---- per-thread roles
     const bool perA = p.kind[0] == BC_PERIODIC, perB = p.kind[2] == BC_PERIODIC;
     const bool inA = a >= 0 && a < nA, inB = b >= 0 && b < nB;
-    const bool valid = (inA || perA) && (inB || perB); // holds a real (possibly wrapped) node
-    const bool wrapped = valid && !(inA && inB);
-    const int aw = inA ? a : (a + nA) % nA;
-    const int bw = inB ? b : (b + nB) % nB;
+    // a window position holds a real node if it is inside the domain or is the
+    // periodic ghost column / row (a = -1, nA; b = -1, nB), whose storage the
+    // owning edge nodes refresh at every store (see store_ghosts)
+    const bool valid = (inA || (perA && (a == -1 || a == nA))) && (inB || (perB && (b == -1 || b == nB)));
     const bool interior = tx >= 1 && tx < TA - 1 && ty >= HB && ty < TB - HB;
     const bool owner = interior && inA && inB;
+    // ghost shift of an owner on a periodic edge: a = 0 -> column nA, a = nA-1 -> column -1
+    const int gA = !perA ? 0 : (a == 0 ? nA : (a == nA - 1 ? -nA : 0));
+    const int gB = (D == 2 || !perB) ? 0 : (b == 0 ? nB : (b == nB - 1 ? -nB : 0));
     // pull-source availability along A/B: source at a-1 (c_a = +1), a+1 (c_a = -1)
     const bool okAm = (a - 1 >= 0) || perA, okAp = (a + 1 < nA) || perA;
     const bool okBm = (D == 2) || (b - 1 >= 0) || perB, okBp = (D == 2) || (b + 1 < nB) || perB;
@@ -482,6 +485,17 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         Real *o = dst + (long long)(c + 1) * p.pstride + (long long)b * p.pitch + a;
 #pragma unroll
         for (int q = 0; q < M; q++) o[q * p.mstride] = out[q];
+        // periodic ghost copies of edge nodes (also the corner ghosts)
+        if (gA | gB) {
+            auto put = [&](int da, int db) {
+                Real *g = o + (long long)db * p.pitch + da;
+#pragma unroll
+                for (int q = 0; q < M; q++) g[q * p.mstride] = out[q];
+            };
+            if (gA) put(gA, 0);
+            if (gB) put(0, gB);
+            if (gA && gB) put(gA, gB);
+        }
     };
 
     for (int it = 0; it < nl; it++) {
@@ -491,15 +505,9 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
 
         Real m[M];
         if (valid) {
-            if (!wrapped) {
-                const Real *st = stage + s * SM::stage_elems + ty * SM::BW + tx + offA;
+            const Real *st = stage + s * SM::stage_elems + ty * SM::BW + tx + offA;
 #pragma unroll
-                for (int q = 0; q < M; q++) m[q] = st[q * (TB * SM::BW)];
-            } else {
-                const Real *g = src + (long long)plane_of(c) * p.pstride + (long long)bw * p.pitch + aw;
-#pragma unroll
-                for (int q = 0; q < M; q++) m[q] = g[q * p.mstride];
-            }
+            for (int q = 0; q < M; q++) m[q] = st[q * (TB * SM::BW)];
         }
         __syncthreads(); // stage s consumed; previous layer's F reads done
         if (tid == 0 && it + S < nl) {
@@ -616,6 +624,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
 struct GridArgs {
     int nA, nB, nC, pitch;
     long long mstride, pstride;
+    int perA, perB; // periodic in-plane axes: write ghost copies (set_moments)
 };
 
 // ABI fp64 [M][nC][nB][nA] (rho, u, Pi) -> internal Real layout (rho - 1).
@@ -628,11 +637,16 @@ __global__ void set_moments_kernel(const double *__restrict__ in, Real *__restri
         const int b = (n / g.nA) % g.nB;
         const int c = n / ((long long)g.nA * g.nB);
         Real *o = buf + (long long)(c + 1) * g.pstride + (long long)b * g.pitch + a;
+        const int gA = !g.perA ? 0 : (a == 0 ? g.nA : (a == g.nA - 1 ? -g.nA : 0));
+        const int gB = !g.perB ? 0 : (b == 0 ? g.nB : (b == g.nB - 1 ? -g.nB : 0));
 #pragma unroll
         for (int q = 0; q < M; q++) {
             double v = in[q * N + n];
             if (q == 0) v -= 1.0;
             o[q * g.mstride] = Real(v);
+            if (gA) o[q * g.mstride + gA] = Real(v);
+            if (gB) o[q * g.mstride + (long long)gB * g.pitch] = Real(v);
+            if (gA && gB) o[q * g.mstride + (long long)gB * g.pitch + gA] = Real(v);
         }
     }
 }

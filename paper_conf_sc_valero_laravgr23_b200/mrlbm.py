@@ -33,7 +33,7 @@ API = ("mrlbm_default_options", "mrlbm_create", "mrlbm_set_moments", "mrlbm_step
        "mrlbm_get_populations", "mrlbm_set_moments_device", "mrlbm_get_moments_device", "mrlbm_sync",
        "mrlbm_check_finite", "mrlbm_query", "mrlbm_launch_count", "mrlbm_time_steps", "mrlbm_destroy",
        "mrlbm_status_string", "mrlbm_last_error", "mrlbm_nccl_unique_id")
-HOST_HELPERS = ("mrlbm_partition", "mrlbm_validate", "mrlbm_kernel_config")
+HOST_HELPERS = ("mrlbm_partition", "mrlbm_validate", "mrlbm_kernel_config", "mrlbm_step_group")
 
 
 class Face(ctypes.Structure):
@@ -79,6 +79,7 @@ def _load():
         "mrlbm_validate": (ctypes.c_int, [ctypes.c_int, i64, i64, i64, ctypes.c_double, ctypes.c_int,
                                           ctypes.POINTER(Boundary), ctypes.c_int]),
         "mrlbm_kernel_config": (ctypes.c_int, [vp, ip, ip, ip, ip, ip, ip, i64p]),
+        "mrlbm_step_group": (ctypes.c_int, [ctypes.POINTER(vp), ctypes.c_int, i64]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -140,6 +141,12 @@ def validate(lattice, nx, ny, nz, tau, regularization="projective", boundary=Non
     b = make_boundary(boundary, D, keep)
     return lib.mrlbm_validate(LATTICES[lattice], nx, ny, nz if D == 3 else 1, float(tau), REGS[regularization],
                               ctypes.byref(b), nranks)
+
+
+def step_group(solvers, n):
+    """Advance a single-process slab group (ranks 0..P-1 created without an NCCL id)."""
+    arr = (ctypes.c_void_p * len(solvers))(*[s._h.value for s in solvers])
+    _check(lib.mrlbm_step_group(arr, len(solvers), int(n)), "mrlbm_step_group")
 
 
 def nccl_unique_id() -> bytes:

@@ -1,0 +1,96 @@
+"""Host-side checks that need no GPU: the C-ABI library loads and exports
+every symbol include/mrlbm.h declares, argument validation, slab partition,
+and the product path fails loudly (no CPU fallback) without a device."""
+import re
+from pathlib import Path
+
+import numpy as np
+import pytest
+
+from paper_conf_sc_valero_laravgr23_b200 import distributed, mrlbm
+
+ROOT = Path(__file__).resolve().parents[1]
+
+
+def header_symbols():
+    txt = (ROOT / "include" / "mrlbm.h").read_text()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return sorted(set(re.findall(r"\b(mrlbm_[a-z_]+)\s*\(", txt)))
+
+
+def test_library_exports_every_declared_symbol():
+    syms = header_symbols()
+    assert len(syms) >= 20
+    for s in syms:
+        assert hasattr(mrlbm.lib, s), s
+    # the binding marshals every one of them
+    assert set(syms) <= set(mrlbm.API) | set(mrlbm.HOST_HELPERS)
+
+
+def test_library_is_built_for_sm100a():
+    import subprocess
+    out = subprocess.run(["cuobjdump", "-lelf", str(mrlbm._LIB_PATH)], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    sass = subprocess.run(["cuobjdump", "-sass", str(mrlbm._LIB_PATH)], capture_output=True, text=True).stdout
+    # the fused step kernels stage their tiles with TMA (UTMALDG) and mbarriers (SYNCS)
+    assert "mrlbm_step_kernel" in sass and "UTMALDG" in sass and "SYNCS" in sass
+
+
+def test_status_strings():
+    assert mrlbm.lib.mrlbm_status_string(0) == b"MRLBM_OK"
+    assert mrlbm.lib.mrlbm_status_string(-7) == b"MRLBM_ERR_BUFFER_SIZE"
+
+
+@pytest.mark.parametrize("n,p", [(10, 1), (10, 3), (1024, 8), (7, 7), (1000, 6)])
+def test_partition_covers_axis(n, p):
+    pieces = [mrlbm.partition(n, p, r) for r in range(p)]
+    assert sum(nl for nl, _ in pieces) == n
+    off = 0
+    for r, (nl, o) in enumerate(pieces):
+        assert o == off and nl >= n // p and nl <= n // p + 1
+        assert (o, nl) == distributed.slab_bounds(n, p, r)
+        off += nl
+
+
+def walls(D):
+    faces = ["x-", "x+", "y-", "y+"] + (["z-", "z+"] if D == 3 else [])
+    return {f: {"kind": "wall"} for f in faces}
+
+
+def test_validation_codes():
+    INV, UNS = -1, -2
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6) == 0
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.5) == INV            # tau <= 1/2 (eq 5)
+    assert mrlbm.validate("D3Q19", 1, 8, 8, 0.6) == INV            # n < 2
+    assert mrlbm.validate("D3Q27", 8, 8, 1, 0.6) == INV            # 3D needs nz >= 2
+    assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, boundary={"x-": {"kind": "wall"}}) == INV  # one-sided periodic
+    b = walls(3)
+    b["y+"] = {"kind": "moving_wall", "u": [0.0, 0.1, 0.0]}       # normal lid velocity
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, boundary=b) == INV
+    b = walls(3)
+    b["z-"] = {"kind": "velocity", "u": [0, 0, 0.01]}              # open face on the sweep axis
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, boundary=b) == UNS
+    b = walls(3)
+    b["x-"] = {"kind": "velocity", "u": [0.01, 0, 0]}
+    b["y+"] = {"kind": "pressure", "rho": 1.0}                      # open faces sharing an edge
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, boundary=b) == UNS
+    b = walls(2)
+    b["x-"] = {"kind": "velocity", "u": [0.01, 0, 0]}
+    b["x+"] = {"kind": "pressure", "rho": 1.0}
+    assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, boundary=b) == 0
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, nranks=8) == INV  # < 2 layers per rank
+
+
+def test_create_fails_loudly_without_gpu():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is present")
+    with pytest.raises(mrlbm.MRLBMError) as e:
+        mrlbm.Solver("D2Q9", 8, 8, 1, 0.6)
+    assert e.value.status == -4  # MRLBM_ERR_CUDA: no silent CPU path
+
+
+def test_slab_cut_and_reassemble():
+    m = np.random.default_rng(0).standard_normal((10, 13, 5, 4))
+    parts = [distributed.slab_of(m, 4, r) for r in range(4)]
+    assert np.array_equal(np.concatenate(parts, axis=1), m)
