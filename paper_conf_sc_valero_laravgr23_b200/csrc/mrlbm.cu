@@ -102,9 +102,12 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile)
     if constexpr (LAT == mr::LAT_D2Q9) {
         return make_variant<LAT, REC, Real, 128, 1, 4, 5>();
     } else {
-        constexpr bool big = LAT == mr::LAT_D3Q27 && sizeof(Real) == 8; // 24 movers x 512 x 8 B
-        if (tile == 1) return make_variant<LAT, REC, Real, 32, 8, 3, 2>();
-        return make_variant<LAT, REC, Real, 32, 16, (big ? 2 : 3), 1>();
+        constexpr bool f64 = sizeof(Real) == 8;
+        // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
+        constexpr bool small_only = LAT == mr::LAT_D3Q27 && f64;
+        if (tile == 0) tile = (LAT == mr::LAT_D3Q19 || small_only) ? 1 : 2;
+        if (tile == 1 || small_only) return make_variant<LAT, REC, Real, 32, 8, (f64 ? 2 : 3), 2>();
+        return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 3), 1>();
     }
 }
 

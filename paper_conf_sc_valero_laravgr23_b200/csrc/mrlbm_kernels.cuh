@@ -305,6 +305,96 @@ template <class L, int k, typename Real> __device__ __forceinline__ void accum(R
     });
 }
 
+// ------------------------------------------------------------ factorised accumulation
+// Values whose zero-ness is known at compile time (absent lattice directions).
+template <bool P, typename Real> struct OV {
+    Real v;
+};
+template <typename Real> struct OV<false, Real> {
+};
+template <bool A, bool B, typename Real> __device__ __forceinline__ auto ov_add(OV<A, Real> a, OV<B, Real> b)
+{
+    if constexpr (A && B) return OV<true, Real>{a.v + b.v};
+    else if constexpr (A) return a;
+    else if constexpr (B) return b;
+    else return OV<false, Real>{};
+}
+template <bool A, bool B, typename Real> __device__ __forceinline__ auto ov_sub(OV<A, Real> a, OV<B, Real> b)
+{
+    if constexpr (A && B) return OV<true, Real>{a.v - b.v};
+    else if constexpr (A) return a;
+    else if constexpr (B) return OV<true, Real>{-b.v};
+    else return OV<false, Real>{};
+}
+// acc += sgn * x  (sgn in {-1, 0, +1}, compile time)
+template <int SG, bool A, typename Real> __device__ __forceinline__ void ov_acc(Real &acc, OV<A, Real> x)
+{
+    if constexpr (A && SG == 1) acc += x.v;
+    else if constexpr (A && SG == -1) acc -= x.v;
+}
+template <class A, class B, class C> struct Tri {
+    A r0;
+    B r1;
+    C r2;
+};
+// 1D moment sums over c in {-1,0,+1}: r0 = sum g, r1 = sum c g, r2 = sum c^2 g
+template <class GM, class G0, class GP> __device__ __forceinline__ auto sums3(GM gm, G0 g0, GP gp)
+{
+    auto r2 = ov_add(gp, gm);
+    auto r1 = ov_sub(gp, gm);
+    auto r0 = ov_add(r2, g0);
+    return Tri<decltype(r0), decltype(r1), decltype(r2)>{r0, r1, r2};
+}
+
+// lattice direction with kernel-axis velocity (ca, cb, cm), or -1
+template <class L> constexpr int dir_of(int ca, int cb, int cm)
+{
+    for (int k = 0; k < L::Q; k++)
+        if (Axes<L>::ca(k) == ca && Axes<L>::cb(k) == cb && Axes<L>::cm(k) == cm) return k;
+    return -1;
+}
+
+// Add the raw moments (sum f, sum c f, sum c c f) of the arrivals G(ia, ib)
+// that move by CM along the sweep axis to acc, sum-factorised: sums over c_a
+// per row c_b, then over c_b; the sweep component c_m = CM enters as a factor.
+template <class L, int CM, typename Real, class GF>
+__device__ __forceinline__ void accum_group(Real (&acc)[L::M], GF &&G)
+{
+    constexpr int D = L::D;
+    using I0 = std::integral_constant<int, 0>;
+    using I1 = std::integral_constant<int, 1>;
+    using I2 = std::integral_constant<int, 2>;
+    // rows: r[ib] over c_a
+    auto rm = sums3(G(I0{}, I0{}), G(I1{}, I0{}), G(I2{}, I0{})); // c_b = -1
+    auto rz = sums3(G(I0{}, I1{}), G(I1{}, I1{}), G(I2{}, I1{})); // c_b = 0
+    auto rp = sums3(G(I0{}, I2{}), G(I1{}, I2{}), G(I2{}, I2{})); // c_b = +1
+    // columns over c_b
+    auto Sbb = ov_add(rp.r0, rm.r0);                 // sum cb^2 f
+    auto Sb = ov_sub(rp.r0, rm.r0);                  // sum cb f
+    auto S = ov_add(Sbb, rz.r0);                     // sum f
+    auto Sa = ov_add(ov_add(rp.r1, rm.r1), rz.r1);   // sum ca f
+    auto Saa = ov_add(ov_add(rp.r2, rm.r2), rz.r2);  // sum ca^2 f
+    auto Sab = ov_sub(rp.r1, rm.r1);                 // sum ca cb f
+    constexpr int CM2 = CM * CM;
+    ov_acc<1>(acc[0], S);
+    ov_acc<1>(acc[1], Sa);                           // j_x (A = x)
+    if constexpr (D == 3) {
+        ov_acc<1>(acc[2], Sb);                       // j_y (B = y)
+        ov_acc<CM>(acc[3], S);                       // j_z (C = z)
+        ov_acc<1>(acc[pslot<3>(0, 0)], Saa);
+        ov_acc<1>(acc[pslot<3>(1, 1)], Sbb);
+        ov_acc<CM2>(acc[pslot<3>(2, 2)], S);
+        ov_acc<1>(acc[pslot<3>(0, 1)], Sab);
+        ov_acc<CM>(acc[pslot<3>(0, 2)], Sa);
+        ov_acc<CM>(acc[pslot<3>(1, 2)], Sb);
+    } else {                                         // 2D: C = y, no B axis
+        ov_acc<CM>(acc[2], S);
+        ov_acc<1>(acc[pslot<2>(0, 0)], Saa);
+        ov_acc<CM2>(acc[pslot<2>(1, 1)], S);
+        ov_acc<CM>(acc[pslot<2>(0, 1)], Sa);
+    }
+}
+
 // ------------------------------------------------------------ step kernel
 template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
     using L = Lattice<LAT>;
@@ -315,8 +405,9 @@ template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
     static constexpr int BW = (TA + AL - 1 + AL - 1) / AL * AL;
     static constexpr size_t box_elems = size_t(L::M) * TB * BW;
     static constexpr size_t stage_elems = (box_elems * sizeof(Real) + 127) / 128 * 128 / sizeof(Real);
-    static constexpr size_t F_elems = size_t(Axes<L>::NMOVE) * NT;
-    static constexpr size_t bytes = (S * stage_elems + F_elems) * sizeof(Real) + S * sizeof(uint64_t) + 128;
+    static constexpr size_t F_elems = size_t(Axes<L>::NMOVE) * NT; // one exchange plane
+    // two exchange planes (alternating layers) -> one __syncthreads per layer
+    static constexpr size_t bytes = (S * stage_elems + 2 * F_elems) * sizeof(Real) + S * sizeof(uint64_t) + 128;
 };
 
 template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB>
@@ -333,7 +424,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     extern __shared__ __align__(128) unsigned char smem_raw[];
     Real *stage = reinterpret_cast<Real *>(smem_raw);
     Real *Fs = stage + S * SM::stage_elems;
-    uint64_t *full = reinterpret_cast<uint64_t *>(Fs + SM::F_elems);
+    uint64_t *full = reinterpret_cast<uint64_t *>(Fs + 2 * SM::F_elems);
 
     const int tid = threadIdx.x;
     const int tx = tid % TA, ty = tid / TA;
@@ -365,8 +456,6 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     const int gA = !perA ? 0 : (a == 0 ? nA : (a == nA - 1 ? -nA : 0));
     const int gB = (D == 2 || !perB) ? 0 : (b == 0 ? nB : (b == nB - 1 ? -nB : 0));
     // pull-source availability along A/B: source at a-1 (c_a = +1), a+1 (c_a = -1)
-    const bool okAm = (a - 1 >= 0) || perA, okAp = (a + 1 < nA) || perA;
-    const bool okBm = (D == 2) || (b - 1 >= 0) || perB, okBp = (D == 2) || (b + 1 < nB) || perB;
     // walls touching this node in-plane (-1 lower face, +1 upper face)
     auto is_wall = [](int k) { return k == BC_WALL || k == BC_MOVING; };
     const int bbA = (a == 0 && is_wall(p.kind[0])) ? -1 : ((a == nA - 1 && is_wall(p.kind[1])) ? 1 : 0);
@@ -509,13 +598,11 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
 #pragma unroll
             for (int q = 0; q < M; q++) m[q] = st[q * (TB * SM::BW)];
         }
-        __syncthreads(); // stage s consumed; previous layer's F reads done
-        if (tid == 0 && it + S < nl) {
-            mbar_expect_tx(&full[s], stage_bytes);
-            tma_load_4d(stage + s * SM::stage_elems, &tmap, &full[s], boxA, b0 + p.padB, 0, plane_of(c + S));
-        }
-
-        // ---- collide + reconstruct (eqs 10-14) and publish in-plane movers
+        // ---- collide + reconstruct (eqs 10-14) and publish the in-plane movers
+        // into exchange plane it & 1 (positions without a node publish zeros,
+        // so pulls need no validity predicate; arrivals into layers that do not
+        // exist land in accumulators that are never stored)
+        Real *Fl = Fs + (it & 1) * SM::F_elems;
         Real fown[Q]; // only the non-moving entries are used after the barrier
         Real rho_own = Real(1);
         if (valid) {
@@ -525,14 +612,21 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
             rho_own = Real(1) + m[0];
             static_for<0, Q>([&](auto kk) {
                 constexpr int k = decltype(kk)::value;
-                if constexpr (X::moving(k)) Fs[X::slot(k) * NT + tid] = fown[k];
+                if constexpr (X::moving(k)) Fl[X::slot(k) * NT + tid] = fown[k];
             });
+        } else {
+#pragma unroll
+            for (int q = 0; q < X::NMOVE; q++) Fl[q * NT + tid] = Real(0);
         }
+        // one barrier per layer: the other exchange plane was last read before
+        // this barrier, and every thread has read stage s
         __syncthreads();
+        if (tid == 0 && it + S < nl) {
+            mbar_expect_tx(&full[s], stage_bytes);
+            tma_load_4d(stage + s * SM::stage_elems, &tmap, &full[s], boxA, b0 + p.padB, 0, plane_of(c + S));
+        }
 
         if (owner) {
-            const bool tgt_lo = (c > 0) || p.lo_nb;      // layer c-1 exists
-            const bool tgt_hi = (c < nC - 1) || p.hi_nb; // layer c+1 exists
             const int bbC = (c == 0 && !p.lo_nb) ? -1 : ((c == nC - 1 && !p.hi_nb) ? 1 : 0);
             auto body = [&](auto open_tag) {
                 constexpr bool OPEN = decltype(open_tag)::value;
@@ -546,27 +640,23 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                 // are accumulated (lower register pressure).
                 auto pull = [&](auto cm_tag) {
                     constexpr int CM = decltype(cm_tag)::value;
-                    static_for<0, Q>([&](auto kk) {
-                        constexpr int k = decltype(kk)::value;
-                        constexpr int ca = X::ca(k), cb = X::cb(k), cm = X::cm(k);
-                        if constexpr (cm == CM) {
-                            bool ok = (cm == 0) || (cm < 0 ? tgt_lo : tgt_hi);
-                            if constexpr (ca > 0) ok = ok && okAm;
-                            if constexpr (ca < 0) ok = ok && okAp;
-                            if constexpr (cb > 0) ok = ok && okBm;
-                            if constexpr (cb < 0) ok = ok && okBp;
-                            if (ok) {
-                                Real v;
-                                if constexpr (X::moving(k)) v = Fs[X::slot(k) * NT + (ty - cb) * TA + (tx - ca)];
-                                else v = fown[k];
-                                if constexpr (OPEN) {
-                                    constexpr int kx = L::c[k][0], ky = L::c[k][1];
-                                    v *= wt(kx, ky);
-                                }
-                                accum<L, k>(acc[cm + 1], v);
+                    auto G = [&](auto iac, auto ibc) {
+                        constexpr int ca = decltype(iac)::value - 1, cb = decltype(ibc)::value - 1;
+                        constexpr int k = dir_of<L>(ca, cb, CM);
+                        if constexpr (k < 0) {
+                            return OV<false, Real>{};
+                        } else {
+                            Real v;
+                            if constexpr (X::moving(k)) v = Fl[X::slot(k) * NT + (ty - cb) * TA + (tx - ca)];
+                            else v = fown[k];
+                            if constexpr (OPEN) {
+                                constexpr int kx = L::c[k][0], ky = L::c[k][1];
+                                v *= wt(kx, ky);
                             }
+                            return OV<true, Real>{v};
                         }
-                    });
+                    };
+                    accum_group<L, CM, Real>(acc[CM + 1], G);
                 };
                 pull(std::integral_constant<int, -1>{});
                 if (c - 1 >= c0 && c - 1 < c1) finalize_store(acc[0], c - 1);
@@ -583,7 +673,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                         const bool xC = (cm != 0) && (cm == bbC);
                         if (xA || xB || xC) {
                             Real v;
-                            if constexpr (X::moving(k)) v = Fs[X::slot(k) * NT + tid];
+                            if constexpr (X::moving(k)) v = Fl[X::slot(k) * NT + tid];
                             else v = fown[k];
                             constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
                             constexpr double wk6 = 6.0 * L::w[k];
