@@ -532,21 +532,38 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     h->tilesA = (h->nA + TA - 3) / (TA - 2);
     h->tilesB = h->D == 3 ? (h->nB + TB - 3) / (TB - 2) : 1;
     a.tilesA = h->tilesA;
-    // segments along C: short enough that the resident CTAs sweep nearby
-    // layers together (their halo re-reads then hit L2) and that there are
-    // >= ~4 waves of CTAs; >= 8 layers so the two halo layers per segment
-    // stay cheap.  MRLBM_SEG overrides (tuning).
+    // Segments along C.  The grid is tiles x segments; pick the segment count
+    // that best fills whole waves of resident CTAs (no tail wave), preferring
+    // longer segments (each segment re-reads one halo layer at each end).
+    // MRLBM_SEG overrides (tuning).
     {
         const long long tiles = (long long)h->tilesA * h->tilesB;
+        int occ = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, h->var.kernel_fn, h->var.TA * h->var.TB, h->var.smem);
+        int nsm = 148;
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        const long long slots = (long long)std::max(occ, 1) * nsm;
         long long seg = env_int("MRLBM_SEG", 0);
-        if (seg <= 0) {
-            const long long target = 148LL * 4 * 4;
-            const long long nseg = std::max<long long>(1, target / std::max<long long>(1, tiles));
-            seg = (h->nC + nseg - 1) / nseg;
-            seg = std::min<long long>(seg, 64);
+        if (seg <= 0 && h->D == 2) {
+            // 2D: short segments keep the resident CTAs on nearby rows, so the
+            // halo columns they share are L2 hits (measured: 24 rows best on C2)
+            seg = 24;
+        } else if (seg <= 0) {
+            // 3D: segment lengths 32..96; best wave fill, ties to the longer
+            double best = -1.0;
+            for (long long sl = std::min<long long>(96, h->nC); sl >= std::min<long long>(32, h->nC); sl--) {
+                const long long ns = (h->nC + sl - 1) / sl;
+                const long long units = tiles * ns;
+                const long long waves = (units + slots - 1) / slots;
+                const double fill = double(units) / double(waves * slots);
+                const double score = fill * (double(sl) / double(sl + 2));
+                if (score > best + 1e-3) {
+                    best = score;
+                    seg = sl;
+                }
+            }
         }
-        seg = std::max<long long>(seg, std::min<long long>(8, h->nC));
-        seg = std::min<long long>(seg, h->nC);
+        seg = std::max<long long>(1, std::min<long long>(seg, h->nC));
         h->seg_len = (int)seg;
         h->nseg = (int)((h->nC + seg - 1) / seg);
     }
