@@ -131,32 +131,46 @@ def cpu_baseline(c, seconds=12.0, max_side=1024):
                       f"sub-domain of {c.name}, {steps} steps in {dt:.1f} s, OpenMP {threads} threads"}
 
 
-def run_reference(args, rank, world):
-    """--impl reference: the CPU oracle (the tier's reference arm) on rank 0."""
-    if rank != 0:
-        return
+def _oracle_sample(c, side, threads):
     import oracle
-    c = build_config(args.config, args.precision, 1)
-    threads = oracle.max_threads()
-    side = args.ref_side
     nx, ny = min(c.nx, side), min(c.ny, side)
     nz = 1 if c.D == 2 else min(c.nz, max(8, side // 8))
     sub = configs.Config(c.name, c.lattice, c.regularization, nx, ny, nz, c.tau, "fp64", c.boundary, c.init, c.U)
     b = {k: dict(v) for k, v in sub.boundary.items()}
     for v in b.values():
-        v.pop("u_profile", None)
+        v.pop("u_profile", None)  # the sample uses a uniform inflow of the config's U
         if v["kind"] == "velocity":
             v["u"] = [c.U, 0, 0]
     o = oracle.Oracle(c.lattice, nx, ny, nz, c.tau, c.regularization, b, threads=threads)
     o.set_moments(sub.initial_moments())
+    return o, (nx, ny, nz), nx * ny * (1 if c.D == 2 else nz)
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle (this tier's reference arm), rank 0 only.
+    Each step is one oracle timestep on a sub-domain of the workload sized so
+    that the K timed steps take about --ref-seconds on this host."""
+    if rank != 0:
+        return
+    import oracle
+    c = build_config(args.config, args.precision, 1)
+    threads = oracle.max_threads()
+    # probe the host rate on a 256^2 (3D: 64^2 x 8) sample, then size the sample
+    o, _, nodes = _oracle_sample(c, 256 if c.D == 2 else 64, threads)
+    t0 = time.perf_counter()
+    o.step(2)
+    rate = 2 * nodes / (time.perf_counter() - t0)  # node updates / s
+    budget = rate * args.ref_seconds / max(1, args.steps)
+    side = int(budget ** 0.5) if c.D == 2 else int((budget / 8) ** 0.5)
+    side = max(16, min(args.ref_side, side))
+    o, dims, nodes = _oracle_sample(c, side, threads)
     o.step(args.warmup)
     t0 = time.perf_counter()
     o.step(args.steps)
     dt = time.perf_counter() - t0
-    nodes = nx * ny * (1 if c.D == 2 else nz)
     v = nodes * args.steps / dt / 1e6
-    sample = (f"{c.lattice}-{c.regularization} {nx}x{ny}{'' if c.D == 2 else 'x' + str(nz)} sub-domain of "
-              f"{c.name} per step, {args.steps} steps in {dt:.2f} s")
+    sample = (f"{c.lattice}-{c.regularization} {'x'.join(map(str, dims[:c.D]))} sub-domain of {c.name} "
+              f"(same faces and tau) per step, {args.steps} steps in {dt:.2f} s, OpenMP {threads} threads")
     line = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
@@ -322,7 +336,8 @@ def main():
     ap.add_argument("--precision", default="fp64", choices=["fp64", "fp32"])
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--ref-side", type=int, default=512, help="reference arm: sample sub-domain side")
+    ap.add_argument("--ref-side", type=int, default=1024, help="reference arm: max sample sub-domain side")
+    ap.add_argument("--ref-seconds", type=float, default=60.0, help="reference arm: target timed seconds")
     args = ap.parse_args()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
