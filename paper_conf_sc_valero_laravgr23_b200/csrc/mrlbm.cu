@@ -100,6 +100,7 @@ template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB> Var
 template <int LAT, bool REC, typename Real> Variant pick(int tile)
 {
     if constexpr (LAT == mr::LAT_D2Q9) {
+        if (tile == 1) return make_variant<LAT, REC, Real, 128, 1, 4, 4>();
         return make_variant<LAT, REC, Real, 128, 1, 4, 5>();
     } else {
         constexpr bool f64 = sizeof(Real) == 8;
