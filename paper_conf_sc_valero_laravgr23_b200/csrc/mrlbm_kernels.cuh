@@ -713,7 +713,8 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     };
     if constexpr (D == 2 && sizeof(Real) == 4) {
         // unrolled by 3: the accumulator roles rotate by renaming, not by moves
-        // (measured: +29% on C2 fp32; slower for fp64, whose unrolled body spills)
+        // (measured: +29% on C2 fp32; slower for fp64, whose unrolled body spills,
+        // and 5x slower for the 3D bodies, which then overflow the instruction cache)
         for (int it = 0; it < nl; it += 3) {
             layer(it, acc[0], acc[1], acc[2]);
             zero(acc[0]);
