@@ -401,6 +401,144 @@ __device__ __forceinline__ void accum_group(Real (&acc)[L::M], GF &&G)
     }
 }
 
+// ------------------------------------------------------------ cold paths (out of line)
+// Kept out of the fused kernel body so that the hot loop stays small enough
+// for the instruction cache; executed only by threads on walls / open faces.
+template <typename Real, int M> struct RVec {
+    Real v[M];
+};
+
+__device__ __forceinline__ double rcp_nr(double x)
+{
+    // branch-free reciprocal: hardware approximation + 3 Newton steps (to ~1 ulp)
+    double r;
+    asm("rcp.approx.ftz.f64 %0, %1;" : "=d"(r) : "d"(x));
+    double e = fma(-x, r, 1.0);
+    r = fma(r, e, r);
+    e = fma(-x, r, 1.0);
+    r = fma(r, e, r);
+    e = fma(-x, r, 1.0);
+    return fma(r, e, r);
+}
+__device__ __forceinline__ float rcp_nr(float x)
+{
+    float r;
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
+    const float e = fmaf(-x, r, 1.0f);
+    return fmaf(r, e, r);
+}
+
+// Halfway bounce-back (push form at the emitting node, R12) with the moving-wall
+// term (R13): the raw-moment increment of the node's own layer.  fl = this
+// thread's slot in the exchange plane (stride NT), fzm / fzp = its non-moving
+// populations with c_m = -1 / +1; wt weights arrivals on an open face (R14).
+template <int LAT, typename Real, int NT>
+__device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *fl, Real fzm, Real fzp, int bbA, int bbB,
+                                                              int bbC, Real rho_own, const StepArgs *p, int nx_in,
+                                                              int ny_in, bool open)
+{
+    using L = Lattice<LAT>;
+    using X = Axes<L>;
+    RVec<Real, L::M> d;
+#pragma unroll
+    for (int q = 0; q < L::M; q++) d.v[q] = Real(0);
+    static_for<0, L::Q>([&](auto kk) {
+        constexpr int k = decltype(kk)::value;
+        constexpr int ca = X::ca(k), cb = X::cb(k), cm = X::cm(k);
+        const bool xA = (ca != 0) && (ca == bbA);
+        const bool xB = (cb != 0) && (cb == bbB);
+        const bool xC = (cm != 0) && (cm == bbC);
+        if (xA || xB || xC) {
+            Real v;
+            if constexpr (X::moving(k)) v = fl[X::slot(k) * NT];
+            else v = (cm < 0) ? fzm : fzp;
+            constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
+            constexpr double wk6 = 6.0 * L::w[k];
+            double cuw = 0.0;
+            auto lid = [&](int face) {
+                if (p->kind[face] == BC_MOVING) cuw += kx * p->uw[face][0] + ky * p->uw[face][1] + kz * p->uw[face][2];
+            };
+            if (xA) lid(ca < 0 ? 0 : 1);
+            if (xB) lid(cb < 0 ? 2 : 3);
+            if (xC) lid(cm < 0 ? 4 : 5);
+            v -= Real(wk6) * rho_own * Real(cuw);
+            constexpr int ko = X::opp(k);
+            if (open) {
+                constexpr int ox = L::c[ko][0], oy = L::c[ko][1];
+                const int cn = ox * nx_in + oy * ny_in;
+                v *= cn > 0 ? Real(0) : (cn < 0 ? Real(2) : Real(1));
+            }
+            accum<L, ko>(d.v, v);
+        }
+    });
+    return d;
+}
+
+// Regularized open face (R14) finalisation from the weighted raw sums s:
+//   velocity face: rho = S0 / (1 - u.n);  pressure face: u.n = 1 - S0 / rho, u_t = 0
+//   Pi = SPi - 6 rho sum_{c.n<0} w H (c.u)   (closed form of the f^neq bounce-back rebuild)
+template <int LAT, typename Real>
+__device__ __forceinline__ RVec<Real, Lattice<LAT>::M> finalize_open(RVec<Real, Lattice<LAT>::M> s, int openF, int nx_in,
+                                                                int ny_in, int cg, int a, int b, int nA, int nB,
+                                                                const StepArgs *p)
+{
+    using L = Lattice<LAT>;
+    constexpr int D = L::D, Q = L::Q, M = L::M;
+    RVec<Real, M> out;
+    const Real S0 = s.v[0];
+    Real u[3] = {Real(0), Real(0), Real(0)};
+    Real drho;
+    if (p->kind[openF] == BC_VELOCITY) {
+        const double *prof = p->open_prof[openF];
+        if (prof) {
+            const long long fi = (openF < 2) ? ((long long)cg * nB + b) : ((long long)cg * nA + a);
+            for (int q = 0; q < D; q++) u[q] = Real(prof[fi * D + q]);
+        } else {
+            for (int q = 0; q < D; q++) u[q] = Real(p->open_u[openF][q]);
+        }
+        const Real un = u[0] * Real(nx_in) + u[1] * Real(ny_in);
+        drho = (S0 + un) / (Real(1) - un);
+    } else {
+        drho = Real(p->open_drho[openF]);
+        const Real rho = Real(1) + drho;
+        const Real un = (drho - S0) / rho;
+        u[0] = un * Real(nx_in);
+        u[1] = un * Real(ny_in);
+    }
+    const Real rho = Real(1) + drho;
+    out.v[0] = drho;
+    for (int q = 0; q < D; q++) out.v[1 + q] = u[q];
+    Real corr[M];
+#pragma unroll
+    for (int q = 0; q < M; q++) corr[q] = Real(0);
+    static_for<0, Q>([&](auto kk) {
+        constexpr int k = decltype(kk)::value;
+        constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
+        constexpr Real wk = Real(L::w[k]);
+        const int cn = kx * nx_in + ky * ny_in;
+        if (cn < 0) {
+            Real cu = Real(kx) * u[0] + Real(ky) * u[1];
+            if constexpr (D == 3) cu += Real(kz) * u[2];
+            const Real t = wk * cu;
+            static_for<0, D>([&](auto qk) {
+                constexpr int q = decltype(qk)::value;
+                static_for<q, D>([&](auto rk) {
+                    constexpr int r = decltype(rk)::value;
+                    constexpr Real H = Real(L::c[k][q] * L::c[k][r]) - ((q == r) ? Real(1.0 / 3.0) : Real(0));
+                    corr[pslot<D>(q, r)] += H * t;
+                });
+            });
+        }
+    });
+#pragma unroll
+    for (int q = 0; q < D; q++)
+#pragma unroll
+        for (int r = q; r < D; r++)
+            out.v[pslot<D>(q, r)] = s.v[pslot<D>(q, r)] - ((q == r) ? S0 * Real(1.0 / 3.0) : Real(0)) -
+                                    Real(6) * rho * corr[pslot<D>(q, r)];
+    return out;
+}
+
 // ------------------------------------------------------------ step kernel
 template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
     using L = Lattice<LAT>;
@@ -503,12 +641,12 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         for (int q = 0; q < M; q++) acc[j][q] = Real(0);
 
     // ---- finalize the completed layer and store it (eqs 1-3; open faces R14)
+    Real *const dst_node = dst + (long long)b * p.pitch + a; // this thread's node in plane 0
     auto finalize_store = [&](const Real (&s)[M], int c) {
         Real out[M];
         const Real S0 = s[0];
         if (openF < 0) {
-            const Real rho = Real(1) + S0;
-            const Real inv = Real(1) / rho;
+            const Real inv = rcp_nr(Real(1) + S0);
             out[0] = S0;
 #pragma unroll
             for (int q = 0; q < D; q++) out[1 + q] = s[1 + q] * inv;
@@ -518,66 +656,14 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                 for (int r = q; r < D; r++)
                     out[pslot<D>(q, r)] = s[pslot<D>(q, r)] - ((q == r) ? S0 * Real(1.0 / 3.0) : Real(0));
         } else {
-            // weighted sums over K0 (x1) and K- (x2) populations:
-            //   S0 = sum wt f = S0~ + 1,  SPi = sum wt H f = acc - delta S0~/3
-            Real u[3] = {Real(0), Real(0), Real(0)};
-            Real drho;
-            const int kind = p.kind[openF];
-            if (kind == BC_VELOCITY) {
-                const double *prof = p.open_prof[openF];
-                if (prof) {
-                    const long long fi = (openF < 2) ? ((long long)(c + p.c_offset) * nB + b)
-                                                     : ((long long)(c + p.c_offset) * nA + a);
+            RVec<Real, M> sv;
 #pragma unroll
-                    for (int q = 0; q < D; q++) u[q] = Real(prof[fi * D + q]);
-                } else {
+            for (int q = 0; q < M; q++) sv.v[q] = s[q];
+            const RVec<Real, M> ov = finalize_open<LAT, Real>(sv, openF, nx_in, ny_in, c + p.c_offset, a, b, nA, nB, &p);
 #pragma unroll
-                    for (int q = 0; q < D; q++) u[q] = Real(p.open_u[openF][q]);
-                }
-                const Real un = u[0] * Real(nx_in) + u[1] * Real(ny_in);
-                drho = (S0 + un) / (Real(1) - un);            // rho = S0 / (1 - u.n)
-            } else {
-                drho = Real(p.open_drho[openF]);
-                const Real rho = Real(1) + drho;
-                const Real un = (drho - S0) / rho;            // u.n = 1 - S0 / rho
-                u[0] = un * Real(nx_in);
-                u[1] = un * Real(ny_in);
-            }
-            const Real rho = Real(1) + drho;
-            out[0] = drho;
-#pragma unroll
-            for (int q = 0; q < D; q++) out[1 + q] = u[q];
-            // Pi = SPi - 2 sum_{K-} H f^eq,odd = SPi - 6 rho sum_{K-} w H (c.u)
-            Real corr[M];
-#pragma unroll
-            for (int q = 0; q < M; q++) corr[q] = Real(0);
-            static_for<0, Q>([&](auto kk) {
-                constexpr int k = decltype(kk)::value;
-                constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
-                constexpr Real wk = Real(L::w[k]);
-                const int cn = kx * nx_in + ky * ny_in;
-                if (cn < 0) {
-                    Real cu = Real(kx) * u[0] + Real(ky) * u[1];
-                    if constexpr (D == 3) cu += Real(kz) * u[2];
-                    const Real t = wk * cu;
-                    static_for<0, D>([&](auto qk) {
-                        constexpr int q = decltype(qk)::value;
-                        static_for<q, D>([&](auto rk) {
-                            constexpr int r = decltype(rk)::value;
-                            constexpr Real H = Real(L::c[k][q] * L::c[k][r]) - ((q == r) ? Real(1.0 / 3.0) : Real(0));
-                            corr[pslot<D>(q, r)] += H * t;
-                        });
-                    });
-                }
-            });
-#pragma unroll
-            for (int q = 0; q < D; q++)
-#pragma unroll
-                for (int r = q; r < D; r++)
-                    out[pslot<D>(q, r)] = s[pslot<D>(q, r)] - ((q == r) ? S0 * Real(1.0 / 3.0) : Real(0)) -
-                                          Real(6) * rho * corr[pslot<D>(q, r)];
+            for (int q = 0; q < M; q++) out[q] = ov.v[q];
         }
-        Real *o = dst + (long long)(c + 1) * p.pstride + (long long)b * p.pitch + a;
+        Real *o = dst_node + (long long)(c + 1) * p.pstride;
 #pragma unroll
         for (int q = 0; q < M; q++) o[q * p.mstride] = out[q];
         // periodic ghost copies of edge nodes (also the corner ghosts)
@@ -669,38 +755,13 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                 if (c - 1 >= c0 && c - 1 < c1) finalize_store(X, c - 1);
                 pull(std::integral_constant<int, 0>{});
                 pull(std::integral_constant<int, 1>{});
-                // halfway bounce-back at walls (push form at the emitting node,
-                // R12) with the moving-wall term (R13)
+                // halfway bounce-back at walls (R12, R13), out of line
                 if (bbA | bbB | bbC) {
-                    static_for<0, Q>([&](auto kk) {
-                        constexpr int k = decltype(kk)::value;
-                        constexpr int ca = X::ca(k), cb = X::cb(k), cm = X::cm(k);
-                        const bool xA = (ca != 0) && (ca == bbA);
-                        const bool xB = (cb != 0) && (cb == bbB);
-                        const bool xC = (cm != 0) && (cm == bbC);
-                        if (xA || xB || xC) {
-                            Real v;
-                            if constexpr (X::moving(k)) v = Fl[X::slot(k) * NT + tid];
-                            else v = fown[k];
-                            constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
-                            constexpr double wk6 = 6.0 * L::w[k];
-                            double cuw = 0.0;
-                            auto lid = [&](int face) {
-                                if (p.kind[face] == BC_MOVING)
-                                    cuw += kx * p.uw[face][0] + ky * p.uw[face][1] + kz * p.uw[face][2];
-                            };
-                            if (xA) lid(ca < 0 ? 0 : 1);
-                            if (xB) lid(cb < 0 ? 2 : 3);
-                            if (xC) lid(cm < 0 ? 4 : 5);
-                            v -= Real(wk6) * rho_own * Real(cuw);
-                            constexpr int ko = X::opp(k);
-                            if constexpr (OPEN) {
-                                constexpr int ox = L::c[ko][0], oy = L::c[ko][1];
-                                v *= wt(ox, oy);
-                            }
-                            accum<L, ko>(Y, v);
-                        }
-                    });
+                    constexpr int kzm = dir_of<L>(0, 0, -1), kzp = dir_of<L>(0, 0, 1);
+                    const RVec<Real, M> d = bounce_back<LAT, Real, NT>(Fl + tid, fown[kzm], fown[kzp], bbA, bbB, bbC,
+                                                                       rho_own, &p, nx_in, ny_in, OPEN);
+#pragma unroll
+                    for (int q = 0; q < M; q++) Y[q] += d.v[q];
                 }
             };
             if (openF >= 0) body(std::true_type{});

@@ -18,7 +18,10 @@ from pathlib import Path
 
 import numpy as np
 
-_LIB_PATH = Path(__file__).resolve().parent / "libmrlbm.so"
+import os
+
+# MRLBM_LIB: load another build of the same library (A/B performance comparisons)
+_LIB_PATH = Path(os.environ.get("MRLBM_LIB") or Path(__file__).resolve().parent / "libmrlbm.so")
 
 LATTICES = {"D2Q9": 0, "D3Q19": 1, "D3Q27": 2}
 REGS = {"projective": 0, "recursive": 1}
