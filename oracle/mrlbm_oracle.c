@@ -19,6 +19,8 @@
  *   equilibrium       eq 4      P:L73 (c_s^2 = 1/3, standard Qian lattices, R1)
  *   Pi^neq            eq 8
  *   projective coll.  eq 9      P:L101 (distribution form)
+ *   BGK collision     Alg. 1 lines 21-25 (eq 5; R2): the
+ *                     paper's standard-representation (ST) reference, NEXT-2
  *   recursive coll.   eqs 10, 12-14  P:L105; recursion of
  *                     Malaspinas [8] (R8), per-component Hermite
  *                     coefficients 1/(a!b!c! c_s^{2n}) (R9), basis per lattice (R10)
@@ -46,7 +48,7 @@
 #define CS2 (1.0 / 3.0) /* lattice speed of sound squared, R1 */
 
 enum { D2Q9 = 0, D3Q19 = 1, D3Q27 = 2 };
-enum { PROJECTIVE = 0, RECURSIVE = 1 };
+enum { PROJECTIVE = 0, RECURSIVE = 1, BGK = 2 };
 enum { PERIODIC = 0, WALL = 1, MOVING_WALL = 2, VELOCITY = 3, PRESSURE = 4 };
 
 typedef struct {
@@ -216,6 +218,14 @@ static void collide_node(const lattice_t *L, int reg, double tau, const double *
             Pneq[a][b] = s;
         }
     const double om = 1.0 - 1.0 / tau;
+    if (reg == BGK) {
+        /* Alg. 1 lines 21-25, the paper's ST reference collision
+         * (single-relaxation-time BGK, eq 5), with the f^eq of eq 4
+         * (R2: the garbled "cu^2" of line 24 is 4.5 (c.u)^2):
+         *   f*_i = f_i (1 - 1/tau) + f^eq_i / tau */
+        for (int i = 0; i < L->Q; i++) fstar[i] = f[i] * om + feq[i] / tau;
+        return;
+    }
     if (reg == PROJECTIVE) {
         /* eq 9: f* = f^eq + (1 - 1/tau) w_i / (2 c_s^4) H2_i : Pi^neq */
         for (int i = 0; i < L->Q; i++) {
