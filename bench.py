@@ -3,6 +3,7 @@ and whole box; achieved HBM GB/s vs peak).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--precision fp64]
   python bench.py --impl reference ...      # the CPU oracle arm (bounded sample)
+  python bench.py --method ST [--collision bgk] ...  # the paper's ST baseline on the GPU
 
 A "step" is one timestep of the whole hot path (load moments -> collide ->
 reconstruct -> stream -> boundaries -> moments -> store; SURVEY 8(a) rows
@@ -11,6 +12,11 @@ a1-a9) over the whole domain.  Default workload = BASELINE.json configs[1]
 For N > 1 (torchrun) every rank owns one 4096 x 4096 y-slab of a 4096 x
 4096N cavity (weak scaling) and exchanges one boundary row of moments per
 step with its neighbours over NCCL.
+
+--method ST runs the same workload in the paper's standard distribution
+representation (Alg. 1: two Q-population lattices, 2 Q w bytes per update,
+BGK collision unless --collision says otherwise) through the same C ABI, so
+that the MR/ST speed-up of the paper is measured on B200.
 
 Timing: W untimed warm-up steps; K steps bracketed by barrier +
 cuda.synchronize, timed with CUDA events on the stream the kernels are
@@ -182,7 +188,8 @@ def run_reference(args, rank, world):
 
 def workload_config(c, world):
     dims = f"{c.nx}x{c.ny}" if c.D == 2 else f"{c.nx}x{c.ny}x{c.nz}"
-    return {"workload": f"{c.name}: {c.lattice} {c.regularization}-regularized "
+    coll = "BGK" if c.regularization == "bgk" else f"{c.regularization}-regularized"
+    return {"workload": f"{c.name}: {c.lattice} {coll} "
                         f"{'lid-driven cavity' if 'y+' in c.boundary and c.boundary['y+']['kind'] == 'moving_wall' else 'flow'} "
                         f"{dims} {c.precision}",
             "lattice": c.lattice, "regularization": c.regularization, "grid": dims, "tau": c.tau,
@@ -192,7 +199,7 @@ def workload_config(c, world):
                   * roofline.WORD[c.precision] > 126e6 else "state fits in L2"}
 
 
-def traffic_from_profiles(c):
+def traffic_from_profiles(c, method="MR"):
     """dram bytes per launch of the fused kernel from the committed ncu summary."""
     p = ROOT / "profiles" / "ncu_summary.json"
     if not p.exists():
@@ -200,6 +207,8 @@ def traffic_from_profiles(c):
     try:
         d = json.loads(p.read_text())
         key = f"{c.name}-{c.lattice}-{c.regularization}-{c.precision}-{c.nx}x{c.ny}x{c.nz if c.D == 3 else 1}"
+        if method != "MR":
+            key = f"{method}-{key}"
         return d.get(key, {}).get("dram_bytes_per_launch")
     except Exception:
         return None
@@ -216,6 +225,17 @@ def run_gpu(args, rank, world, local_rank):
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=dev)
     c = build_config(args.config, args.precision, world)
+    st = args.method == "ST"
+    if st:
+        if world > 1:
+            raise SystemExit("--method ST runs on one GPU (the distribution representation is single-rank)")
+        # the paper's ST reference collides with BGK (Alg. 1); --collision overrides
+        c.regularization = args.collision or "bgk"
+        for v in c.boundary.values():
+            if v["kind"] in ("velocity", "pressure"):
+                raise SystemExit("--method ST: open faces are not implemented for the distribution representation")
+    elif args.collision:
+        c.regularization = args.collision
     nccl_id = None
     if world > 1:
         idt = torch.zeros(128, dtype=torch.uint8, device=dev)
@@ -225,7 +245,8 @@ def run_gpu(args, rank, world, local_rank):
         nccl_id = bytes(idt.cpu().numpy().tobytes())
     stream = torch.cuda.Stream(device=dev)
     s = mrlbm.Solver(c.lattice, c.nx, c.ny, c.nz, c.tau, c.regularization, c.boundary, precision=c.precision,
-                     device=local_rank, stream=stream.cuda_stream, rank=rank, nranks=world, nccl_id=nccl_id)
+                     device=local_rank, stream=stream.cuda_stream, rank=rank, nranks=world, nccl_id=nccl_id,
+                     representation="distributions" if st else "moments")
     # initial state: this rank's slab of the seeded initial moments
     m0 = c.initial_moments()
     sl = slice(s.offset, s.offset + s.n_local)
@@ -299,14 +320,14 @@ def run_gpu(args, rank, world, local_rank):
 
     # roofline of the dominant (fused step) kernel: algorithmic bytes 2 M w per node
     peak, peak_src = load_peaks()
-    bpl = roofline.bytes_per_lup(c.lattice, "MR", c.precision)
+    bpl = roofline.bytes_per_lup(c.lattice, "ST" if st else "MR", c.precision)
     launches_per_step = max(1, round(launches / args.steps))
     achieved = nodes_local * bpl / (ms_step * 1e-3) / 1e9
-    tr = traffic_from_profiles(c)
+    tr = traffic_from_profiles(c, args.method)
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64" if c.precision == "fp64" else "f32", "data": "synthetic",
-            "config": workload_config(c, world),
+            "config": dict(workload_config(c, world), method=args.method),
             "per_gpu_mlups": value / world,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": tr, "peak_source": peak_src,
@@ -334,6 +355,10 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C2", choices=list(configs.ALL))
     ap.add_argument("--precision", default="fp64", choices=["fp64", "fp32"])
+    ap.add_argument("--method", default="MR", choices=["MR", "ST"],
+                    help="MR = the paper's moment representation (default); ST = its distribution baseline")
+    ap.add_argument("--collision", default=None, choices=["projective", "recursive", "bgk"],
+                    help="override the collision (ST default: bgk, the paper's Alg. 1)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--ref-side", type=int, default=1024, help="reference arm: max sample sub-domain side")

@@ -44,8 +44,24 @@ typedef struct mrlbm_ctx *mrlbm_t; /* opaque; owns all device memory it allocate
 typedef enum { MRLBM_D2Q9 = 0, MRLBM_D3Q19 = 1, MRLBM_D3Q27 = 2 } mrlbm_lattice;
 
 /* projective: eqs 8-11; recursive: eqs 8, 10, 12-14
- * with Malaspinas' recursion [8] (R8) and the per-lattice basis R10. */
-typedef enum { MRLBM_PROJECTIVE = 0, MRLBM_RECURSIVE = 1 } mrlbm_regularization;
+ * with Malaspinas' recursion [8] (R8) and the per-lattice basis R10.
+ * BGK: the single-relaxation-time collision of the paper's standard reference
+ * (Alg. 1 lines 21-25, eq 4 per R2); it is not moment-closed, so it
+ * exists only with MRLBM_DISTRIBUTIONS (MRLBM_ERR_UNSUPPORTED with MOMENTS). */
+typedef enum { MRLBM_PROJECTIVE = 0, MRLBM_RECURSIVE = 1, MRLBM_BGK = 2 } mrlbm_regularization;
+
+/* State representation.
+ *   MOMENTS       (default) the paper's method (MR, Alg. 2): M moments per node,
+ *                 2 M w bytes per lattice update (Table 2).
+ *   DISTRIBUTIONS the paper's comparison baseline (ST, Alg. 1): Q
+ *                 pre-collision populations per node in two lattices, 2 Q w
+ *                 bytes per update; one push kernel per step (collide + stream,
+ *                 walls as the MR path).  Single rank; periodic / wall /
+ *                 moving-wall faces only (open faces: MRLBM_ERR_UNSUPPORTED).
+ * Both expose the same state through the same calls (moments = eqs 1-3 of the
+ * pre-collision populations) and give the same trajectory for the regularized
+ * collisions up to rounding. */
+typedef enum { MRLBM_MOMENTS = 0, MRLBM_DISTRIBUTIONS = 1 } mrlbm_representation;
 
 /* Arithmetic and storage precision of the device state.  FP64 is the paper's
  * (P:L257); FP32 stores rho - 1 and shifted populations (R16). */
@@ -86,12 +102,14 @@ typedef struct {
     int rank, nranks;          /* z-slab decomposition (2D: y-slabs); default 0, 1 */
     const void *nccl_unique_id;/* 128-byte ncclUniqueId for nranks > 1 (one GPU per
                                   rank); NULL with nranks > 1 = slab-group mode */
+    mrlbm_representation representation; /* default MOMENTS */
 } mrlbm_options;
 
 typedef int mrlbm_status;
 #define MRLBM_OK 0
 #define MRLBM_ERR_INVALID_ARGUMENT -1 /* tau <= 1/2, n < 2, D2Q9 with nz != 1, one-sided periodic, bad kind */
-#define MRLBM_ERR_UNSUPPORTED -2      /* open faces sharing an edge, open face on the marching axis */
+#define MRLBM_ERR_UNSUPPORTED -2      /* open faces sharing an edge, open face on the marching axis;
+                                         BGK with MOMENTS; DISTRIBUTIONS with open faces or nranks > 1 */
 #define MRLBM_ERR_OUT_OF_MEMORY -3
 #define MRLBM_ERR_CUDA -4
 #define MRLBM_ERR_NCCL -5
@@ -125,6 +143,12 @@ mrlbm_status mrlbm_get_moments(mrlbm_t h, double *dst, int64_t count);
 /* Post-collision populations f* of the current state (eqs 9 / 14; R17),
  * [Q][nz_local][ny][nx] fp64 on host.  count must equal Q * N_local. */
 mrlbm_status mrlbm_get_populations(mrlbm_t h, double *dst, int64_t count);
+
+/* Set the state from PRE-collision populations f, [Q][nz_local][ny][nx] fp64
+ * host, count = Q * N_local.  DISTRIBUTIONS stores them as they are.  MOMENTS
+ * stores their moments (eqs 1-3): the regularized collisions read only those
+ * (P:L49), so the trajectory is the same.  Synchronous. */
+mrlbm_status mrlbm_set_populations(mrlbm_t h, const double *src, int64_t count);
 
 /* Device-side variants for zero-copy I/O: dst/src are DEVICE pointers to fp64
  * arrays in the host layout above; enqueued on the handle's stream. */
@@ -171,9 +195,15 @@ mrlbm_status mrlbm_step_group(mrlbm_t *handles, int n_handles, int64_t n);
 mrlbm_status mrlbm_partition(int64_t n, int nranks, int rank, int64_t *n_local, int64_t *offset);
 mrlbm_status mrlbm_validate(mrlbm_lattice lattice, int64_t nx, int64_t ny, int64_t nz, double tau,
                             mrlbm_regularization reg, const mrlbm_boundary *boundary, int nranks);
+/* The same for a given representation (mrlbm_validate = MOMENTS). */
+mrlbm_status mrlbm_validate_repr(mrlbm_lattice lattice, int64_t nx, int64_t ny, int64_t nz, double tau,
+                                 mrlbm_regularization reg, const mrlbm_boundary *boundary, int nranks,
+                                 mrlbm_representation representation);
 
 /* Fused-kernel launch configuration of a handle (tile TA x TB threads, TMA
- * stages S, sweep segment length, grid, dynamic shared memory bytes). */
+ * stages S, sweep segment length, grid, dynamic shared memory bytes).  For
+ * DISTRIBUTIONS: TA = threads per block along x, TB = 1, S = 0, seg_len = 1,
+ * grid_x = blocks along x, grid_y = ny * nz, smem 0. */
 mrlbm_status mrlbm_kernel_config(mrlbm_t h, int *TA, int *TB, int *S, int *seg_len, int *grid_x, int *grid_y,
                                  int64_t *smem_bytes);
 

@@ -6,6 +6,9 @@
 // CUDA graphs, and for nranks > 1 exchanges one boundary plane of moments per
 // step with each z-slab neighbour through NCCL send/recv on a communication
 // stream, overlapped with the interior update.
+// With MRLBM_DISTRIBUTIONS the same handle runs the paper's standard
+// distribution representation (ST, Alg. 1) instead: two Q-population lattices
+// and the push kernel of st_kernels.cuh (the comparison baseline, NEXT-2).
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
@@ -20,6 +23,7 @@
 
 #include "../../include/mrlbm.h"
 #include "mrlbm_kernels.cuh"
+#include "st_kernels.cuh"
 
 namespace {
 
@@ -125,6 +129,62 @@ Variant select_variant(int lat, int reg, int prec, int tile)
 #undef MR_SEL
 }
 
+// ---- distribution representation (ST) dispatch
+struct StVariant {
+    int BX;
+    void (*step)(const mr::StArgs &, dim3, cudaStream_t);
+    void (*set)(const double *, void *, mr::StGrid, cudaStream_t);
+    void (*set_pops)(const double *, void *, mr::StGrid, cudaStream_t);
+    void (*get)(const void *, double *, mr::StGrid, cudaStream_t);
+    void (*pops)(const void *, double *, mr::StGrid, double, double, cudaStream_t);
+    void (*finite)(const void *, mr::StGrid, int *, cudaStream_t);
+    const void *kernel_fn;
+};
+
+template <int LAT, int COLL, typename Real> StVariant make_st()
+{
+    constexpr int BX = 128;
+    StVariant v;
+    v.BX = BX;
+    v.kernel_fn = (const void *)mr::st_step_kernel<LAT, COLL, Real, BX>;
+    v.step = [](const mr::StArgs &a, dim3 grid, cudaStream_t st) {
+        mr::st_step_kernel<LAT, COLL, Real, BX><<<grid, BX, 0, st>>>(a);
+    };
+    v.set = [](const double *in, void *buf, mr::StGrid g, cudaStream_t st) {
+        mr::st_set_moments_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(in, (Real *)buf, g);
+    };
+    v.set_pops = [](const double *in, void *buf, mr::StGrid g, cudaStream_t st) {
+        mr::st_set_populations_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(in, (Real *)buf, g);
+    };
+    v.get = [](const void *buf, double *out, mr::StGrid g, cudaStream_t st) {
+        mr::st_get_moments_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>((const Real *)buf, out, g);
+    };
+    v.pops = [](const void *buf, double *out, mr::StGrid g, double omega, double inv_tau, cudaStream_t st) {
+        mr::st_populations_kernel<LAT, COLL, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(
+            (const Real *)buf, out, g, omega, inv_tau);
+    };
+    v.finite = [](const void *buf, mr::StGrid g, int *flag, cudaStream_t st) {
+        mr::st_finite_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>((const Real *)buf, g, flag);
+    };
+    return v;
+}
+
+template <int LAT> StVariant pick_st(int coll, bool f32)
+{
+    if (coll == MRLBM_BGK) return f32 ? make_st<LAT, mr::COLL_BGK, float>() : make_st<LAT, mr::COLL_BGK, double>();
+    if (coll == MRLBM_RECURSIVE)
+        return f32 ? make_st<LAT, mr::COLL_RECURSIVE, float>() : make_st<LAT, mr::COLL_RECURSIVE, double>();
+    return f32 ? make_st<LAT, mr::COLL_PROJECTIVE, float>() : make_st<LAT, mr::COLL_PROJECTIVE, double>();
+}
+
+StVariant select_st(int lat, int coll, int prec)
+{
+    const bool F = prec == MRLBM_FP32;
+    if (lat == MRLBM_D2Q9) return pick_st<mr::LAT_D2Q9>(coll, F);
+    if (lat == MRLBM_D3Q19) return pick_st<mr::LAT_D3Q19>(coll, F);
+    return pick_st<mr::LAT_D3Q27>(coll, F);
+}
+
 int env_int(const char *name, int dflt)
 {
     const char *v = getenv(name);
@@ -181,6 +241,11 @@ struct mrlbm_ctx {
     cudaGraphExec_t graph[2] = {nullptr, nullptr};
     int graph_steps = 0;
     int64_t kernels = 0;
+    // distribution representation (ST)
+    int repr = MRLBM_MOMENTS;
+    StVariant sv;
+    mr::StArgs st_base;
+    mr::StGrid st_grid;
 };
 
 namespace {
@@ -222,7 +287,14 @@ void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st)
 mrlbm_status enqueue_one_step(mrlbm_ctx *h, cudaStream_t st)
 {
     const int src = h->cur;
-    if (h->nranks == 1) {
+    if (h->repr == MRLBM_DISTRIBUTIONS) {
+        mr::StArgs a = h->st_base;
+        a.src = h->buf[src];
+        a.dst = h->buf[1 - src];
+        dim3 grid((unsigned)((h->st_grid.nx + h->sv.BX - 1) / h->sv.BX), (unsigned)h->st_grid.ny, (unsigned)h->st_grid.nz);
+        h->sv.step(a, grid, st);
+        h->kernels++;
+    } else if (h->nranks == 1) {
         launch_range(h, src, 0, h->nC, st);
     } else {
         // halo exchange of the boundary planes of the current state, overlapped
@@ -325,8 +397,21 @@ mrlbm_status mrlbm_partition(int64_t n, int nranks, int rank, int64_t *n_local, 
 mrlbm_status mrlbm_validate(mrlbm_lattice lattice, int64_t nx, int64_t ny, int64_t nz, double tau,
                             mrlbm_regularization reg, const mrlbm_boundary *bnd, int nranks)
 {
+    return mrlbm_validate_repr(lattice, nx, ny, nz, tau, reg, bnd, nranks, MRLBM_MOMENTS);
+}
+
+mrlbm_status mrlbm_validate_repr(mrlbm_lattice lattice, int64_t nx, int64_t ny, int64_t nz, double tau,
+                                 mrlbm_regularization reg, const mrlbm_boundary *bnd, int nranks,
+                                 mrlbm_representation repr)
+{
     if (lattice < MRLBM_D2Q9 || lattice > MRLBM_D3Q27) return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown lattice");
-    if (reg != MRLBM_PROJECTIVE && reg != MRLBM_RECURSIVE) return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown regularization");
+    if (repr != MRLBM_MOMENTS && repr != MRLBM_DISTRIBUTIONS) return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown representation");
+    if (reg != MRLBM_PROJECTIVE && reg != MRLBM_RECURSIVE && reg != MRLBM_BGK)
+        return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown regularization");
+    if (reg == MRLBM_BGK && repr == MRLBM_MOMENTS)
+        return fail(MRLBM_ERR_UNSUPPORTED, "BGK is not moment-closed: use the distribution representation");
+    if (repr == MRLBM_DISTRIBUTIONS && nranks != 1)
+        return fail(MRLBM_ERR_UNSUPPORTED, "the distribution representation runs on one rank");
     if (!(tau > 0.5) || !std::isfinite(tau)) return fail(MRLBM_ERR_INVALID_ARGUMENT, "tau must be > 1/2 (eq 5)");
     const int D = lattice == MRLBM_D2Q9 ? 2 : 3;
     if (nx < 2 || ny < 2) return fail(MRLBM_ERR_INVALID_ARGUMENT, "nx, ny must be >= 2");
@@ -353,6 +438,10 @@ mrlbm_status mrlbm_validate(mrlbm_lattice lattice, int64_t nx, int64_t ny, int64
             return fail(MRLBM_ERR_INVALID_ARGUMENT, "2D moving-wall velocity has a z component");
         if (f.kind == MRLBM_PRESSURE && !(f.rho > 0)) return fail(MRLBM_ERR_INVALID_ARGUMENT, "pressure face needs rho > 0");
     }
+    if (repr == MRLBM_DISTRIBUTIONS)
+        for (int F = 0; F < 2 * D; F++)
+            if (is_open(bnd->face[F].kind))
+                return fail(MRLBM_ERR_UNSUPPORTED, "open faces are not implemented for the distribution representation");
     const int march = D == 3 ? 2 : 1;
     if (is_open(bnd->face[2 * march].kind) || is_open(bnd->face[2 * march + 1].kind))
         return fail(MRLBM_ERR_UNSUPPORTED, "open faces on the marching/slab axis are not supported");
@@ -373,7 +462,7 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     mrlbm_default_options(&o);
     if (opt) o = *opt;
     if (o.precision != MRLBM_FP64 && o.precision != MRLBM_FP32) return fail(MRLBM_ERR_INVALID_ARGUMENT, "precision");
-    mrlbm_status st = mrlbm_validate(lattice, nx, ny, nz, tau, reg, boundary, o.nranks);
+    mrlbm_status st = mrlbm_validate_repr(lattice, nx, ny, nz, tau, reg, boundary, o.nranks, o.representation);
     if (st) return st;
     if (o.rank < 0 || o.rank >= o.nranks) return fail(MRLBM_ERR_INVALID_ARGUMENT, "rank out of range");
 
@@ -381,7 +470,7 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     if (o.device >= 0) MR_CUDA(cudaSetDevice(o.device));
     int dev = 0;
     MR_CUDA(cudaGetDevice(&dev));
-    if (!encode) return fail(MRLBM_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    if (!encode && o.representation == MRLBM_MOMENTS) return fail(MRLBM_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
 
     mrlbm_ctx *h = new mrlbm_ctx();
     h->device = dev;
@@ -399,6 +488,7 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     h->omega = 1.0 - 1.0 / tau;
     h->rank = o.rank;
     h->nranks = o.nranks;
+    h->repr = o.representation;
     if (boundary) h->bnd = *boundary;
     else memset(&h->bnd, 0, sizeof(h->bnd)); // all periodic
 
@@ -441,6 +531,51 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
         cudaEventCreateWithFlags(&h->ev_comm, cudaEventDisableTiming) != cudaSuccess ||
         cudaEventCreate(&h->ev_t0) != cudaSuccess || cudaEventCreate(&h->ev_t1) != cudaSuccess)
         return cleanup_fail(fail(MRLBM_ERR_CUDA, "stream/event create"));
+
+    if (h->repr == MRLBM_DISTRIBUTIONS) {
+        // two lattices of Q shifted populations [q][z][y][x], rows 128-B aligned
+        mr::StGrid &g = h->st_grid;
+        g.nx = (int)nx;
+        g.ny = (int)ny;
+        g.nz = (int)h->gn[2];
+        g.pitch = (int)((nx + 31) / 32 * 32);
+        g.plane = (long long)g.ny * g.pitch;
+        g.qstride = (long long)g.nz * g.plane;
+        h->buf_bytes = (size_t)h->Q * g.qstride * h->wbytes;
+        for (int i = 0; i < 2; i++) {
+            if (cudaMalloc(&h->buf[i], h->buf_bytes) != cudaSuccess) {
+                cudaGetLastError();
+                return cleanup_fail(fail(MRLBM_ERR_OUT_OF_MEMORY, "state allocation failed"));
+            }
+            // zeros = shifted populations of the rest state f = w
+            if (cudaMemsetAsync(h->buf[i], 0, h->buf_bytes, h->stream) != cudaSuccess)
+                return cleanup_fail(fail(MRLBM_ERR_CUDA, "memset"));
+        }
+        if (cudaMalloc(&h->flag, sizeof(int)) != cudaSuccess) return cleanup_fail(fail(MRLBM_ERR_OUT_OF_MEMORY, "flag"));
+        h->sv = select_st(lattice, reg, o.precision);
+        mr::StArgs &a = h->st_base;
+        memset(&a, 0, sizeof(a));
+        a.nx = g.nx;
+        a.ny = g.ny;
+        a.nz = g.nz;
+        a.pitch = g.pitch;
+        a.plane = g.plane;
+        a.qstride = g.qstride;
+        a.omega = h->omega;
+        a.inv_tau = 1.0 / tau;
+        for (int F = 0; F < 6; F++) {
+            const mrlbm_face &f = h->bnd.face[F];
+            a.kind[F] = (F < 2 * h->D) ? (int)f.kind : mr::BC_PERIODIC;
+            for (int q = 0; q < 3; q++) a.uw[F][q] = (F < 2 * h->D && f.kind == MRLBM_MOVING_WALL) ? f.u[q] : 0.0;
+        }
+        h->tilesA = (g.nx + h->sv.BX - 1) / h->sv.BX;
+        h->tilesB = 1;
+        h->seg_len = 1;
+        h->nseg = g.ny * g.nz;
+        if (cudaStreamSynchronize(h->stream) != cudaSuccess) return cleanup_fail(fail(MRLBM_ERR_CUDA, "sync"));
+        *out = h;
+        return MRLBM_OK;
+    }
 
     for (int i = 0; i < 2; i++) {
         if (cudaMalloc(&h->buf[i], h->buf_bytes) != cudaSuccess) {
@@ -614,7 +749,8 @@ mrlbm_status mrlbm_set_moments_device(mrlbm_t h, const double *src_dev, int64_t 
 {
     if (!h || !src_dev) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
     if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
-    h->var.set(src_dev, node0(h, h->cur), grid_args(h), h->stream);
+    if (h->repr == MRLBM_DISTRIBUTIONS) h->sv.set(src_dev, h->buf[h->cur], h->st_grid, h->stream);
+    else h->var.set(src_dev, node0(h, h->cur), grid_args(h), h->stream);
     MR_CUDA(cudaGetLastError());
     return MRLBM_OK;
 }
@@ -623,7 +759,8 @@ mrlbm_status mrlbm_get_moments_device(mrlbm_t h, double *dst_dev, int64_t count)
 {
     if (!h || !dst_dev) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
     if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
-    h->var.get(node0(h, h->cur), dst_dev, grid_args(h), h->stream);
+    if (h->repr == MRLBM_DISTRIBUTIONS) h->sv.get(h->buf[h->cur], dst_dev, h->st_grid, h->stream);
+    else h->var.get(node0(h, h->cur), dst_dev, grid_args(h), h->stream);
     MR_CUDA(cudaGetLastError());
     return MRLBM_OK;
 }
@@ -660,9 +797,51 @@ mrlbm_status mrlbm_get_populations(mrlbm_t h, double *dst, int64_t count)
     if (count != (int64_t)h->Q * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != Q * N_local");
     mrlbm_status s = ensure_io(h, (size_t)count * sizeof(double));
     if (s) return s;
-    h->var.pops(node0(h, h->cur), h->io, grid_args(h), h->omega, h->stream);
+    if (h->repr == MRLBM_DISTRIBUTIONS) h->sv.pops(h->buf[h->cur], h->io, h->st_grid, h->omega, 1.0 / h->tau, h->stream);
+    else h->var.pops(node0(h, h->cur), h->io, grid_args(h), h->omega, h->stream);
     MR_CUDA(cudaGetLastError());
     MR_CUDA(cudaMemcpyAsync(dst, h->io, (size_t)count * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    MR_CUDA(cudaStreamSynchronize(h->stream));
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_set_populations(mrlbm_t h, const double *src, int64_t count)
+{
+    if (!h || !src) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
+    if (h->group_mode) return fail(MRLBM_ERR_UNSUPPORTED, "set_populations on a slab-group handle");
+    const int64_t N = local_nodes(h);
+    if (count != (int64_t)h->Q * N) return fail(MRLBM_ERR_BUFFER_SIZE, "count != Q * N_local");
+    mrlbm_status s = ensure_io(h, (size_t)(h->Q + h->M) * N * sizeof(double));
+    if (s) return s;
+    MR_CUDA(cudaMemcpyAsync(h->io, src, (size_t)count * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+    if (h->repr == MRLBM_DISTRIBUTIONS) {
+        h->sv.set_pops(h->io, h->buf[h->cur], h->st_grid, h->stream);
+    } else {
+        // moments of f (eqs 1-3), computed by the ST moment kernel over a dense
+        // [Q][N] view of the staging buffer, then stored as the MR state
+        mr::StGrid g;
+        g.nx = h->nA;
+        g.ny = h->nB * h->nC;
+        g.nz = 1;
+        g.pitch = h->nA;
+        g.plane = (long long)g.ny * g.pitch;
+        g.qstride = g.plane;
+        double *mom = h->io + (size_t)h->Q * N;
+        const int lat = h->lattice;
+        if (lat == MRLBM_D2Q9) {
+            mr::st_set_populations_kernel<mr::LAT_D2Q9, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, h->io, g);
+            mr::st_get_moments_kernel<mr::LAT_D2Q9, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, mom, g);
+        } else if (lat == MRLBM_D3Q19) {
+            mr::st_set_populations_kernel<mr::LAT_D3Q19, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, h->io, g);
+            mr::st_get_moments_kernel<mr::LAT_D3Q19, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, mom, g);
+        } else {
+            mr::st_set_populations_kernel<mr::LAT_D3Q27, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, h->io, g);
+            mr::st_get_moments_kernel<mr::LAT_D3Q27, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, mom, g);
+        }
+        MR_CUDA(cudaGetLastError());
+        h->var.set(mom, node0(h, h->cur), grid_args(h), h->stream);
+    }
+    MR_CUDA(cudaGetLastError());
     MR_CUDA(cudaStreamSynchronize(h->stream));
     return MRLBM_OK;
 }
@@ -717,7 +896,8 @@ mrlbm_status mrlbm_check_finite(mrlbm_t h)
 {
     if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
     MR_CUDA(cudaMemsetAsync(h->flag, 0, sizeof(int), h->stream));
-    h->var.finite(node0(h, h->cur), grid_args(h), h->flag, h->stream);
+    if (h->repr == MRLBM_DISTRIBUTIONS) h->sv.finite(h->buf[h->cur], h->st_grid, h->flag, h->stream);
+    else h->var.finite(node0(h, h->cur), grid_args(h), h->flag, h->stream);
     int v = 0;
     MR_CUDA(cudaMemcpyAsync(&v, h->flag, sizeof(int), cudaMemcpyDeviceToHost, h->stream));
     MR_CUDA(cudaStreamSynchronize(h->stream));
@@ -809,6 +989,16 @@ mrlbm_status mrlbm_kernel_config(mrlbm_t h, int *TA, int *TB, int *S, int *seg_l
                                  int64_t *smem_bytes)
 {
     if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
+    if (h->repr == MRLBM_DISTRIBUTIONS) {
+        if (TA) *TA = h->sv.BX;
+        if (TB) *TB = 1;
+        if (S) *S = 0;
+        if (seg_len) *seg_len = 1;
+        if (grid_x) *grid_x = h->tilesA;
+        if (grid_y) *grid_y = h->nseg;
+        if (smem_bytes) *smem_bytes = 0;
+        return MRLBM_OK;
+    }
     if (TA) *TA = h->var.TA;
     if (TB) *TB = h->var.TB;
     if (S) *S = h->var.S;

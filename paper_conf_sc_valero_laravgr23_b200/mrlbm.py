@@ -24,7 +24,8 @@ import os
 _LIB_PATH = Path(os.environ.get("MRLBM_LIB") or Path(__file__).resolve().parent / "libmrlbm.so")
 
 LATTICES = {"D2Q9": 0, "D3Q19": 1, "D3Q27": 2}
-REGS = {"projective": 0, "recursive": 1}
+REGS = {"projective": 0, "recursive": 1, "bgk": 2}
+REPRS = {"moments": 0, "distributions": 1}
 PRECISIONS = {"fp64": 0, "fp32": 1}
 BC = {"periodic": 0, "wall": 1, "moving_wall": 2, "velocity": 3, "pressure": 4}
 FACES = ("x-", "x+", "y-", "y+", "z-", "z+")
@@ -35,8 +36,8 @@ M_OF = {"D2Q9": 6, "D3Q19": 10, "D3Q27": 10}
 API = ("mrlbm_default_options", "mrlbm_create", "mrlbm_set_moments", "mrlbm_step", "mrlbm_get_moments",
        "mrlbm_get_populations", "mrlbm_set_moments_device", "mrlbm_get_moments_device", "mrlbm_sync",
        "mrlbm_check_finite", "mrlbm_query", "mrlbm_launch_count", "mrlbm_time_steps", "mrlbm_destroy",
-       "mrlbm_status_string", "mrlbm_last_error", "mrlbm_nccl_unique_id")
-HOST_HELPERS = ("mrlbm_partition", "mrlbm_validate", "mrlbm_kernel_config", "mrlbm_step_group")
+       "mrlbm_status_string", "mrlbm_last_error", "mrlbm_nccl_unique_id", "mrlbm_set_populations")
+HOST_HELPERS = ("mrlbm_partition", "mrlbm_validate", "mrlbm_validate_repr", "mrlbm_kernel_config", "mrlbm_step_group")
 
 
 class Face(ctypes.Structure):
@@ -50,7 +51,8 @@ class Boundary(ctypes.Structure):
 
 class Options(ctypes.Structure):
     _fields_ = [("precision", ctypes.c_int), ("device", ctypes.c_int), ("cuda_stream", ctypes.c_void_p),
-                ("rank", ctypes.c_int), ("nranks", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p)]
+                ("rank", ctypes.c_int), ("nranks", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p),
+                ("representation", ctypes.c_int)]
 
 
 def _load():
@@ -66,6 +68,7 @@ def _load():
         "mrlbm_set_moments": (ctypes.c_int, [vp, dp, i64]),
         "mrlbm_get_moments": (ctypes.c_int, [vp, dp, i64]),
         "mrlbm_get_populations": (ctypes.c_int, [vp, dp, i64]),
+        "mrlbm_set_populations": (ctypes.c_int, [vp, dp, i64]),
         "mrlbm_set_moments_device": (ctypes.c_int, [vp, vp, i64]),
         "mrlbm_get_moments_device": (ctypes.c_int, [vp, vp, i64]),
         "mrlbm_step": (ctypes.c_int, [vp, i64]),
@@ -81,6 +84,8 @@ def _load():
         "mrlbm_partition": (ctypes.c_int, [i64, ctypes.c_int, ctypes.c_int, i64p, i64p]),
         "mrlbm_validate": (ctypes.c_int, [ctypes.c_int, i64, i64, i64, ctypes.c_double, ctypes.c_int,
                                           ctypes.POINTER(Boundary), ctypes.c_int]),
+        "mrlbm_validate_repr": (ctypes.c_int, [ctypes.c_int, i64, i64, i64, ctypes.c_double, ctypes.c_int,
+                                               ctypes.POINTER(Boundary), ctypes.c_int, ctypes.c_int]),
         "mrlbm_kernel_config": (ctypes.c_int, [vp, ip, ip, ip, ip, ip, ip, i64p]),
         "mrlbm_step_group": (ctypes.c_int, [ctypes.POINTER(vp), ctypes.c_int, i64]),
     }
@@ -137,13 +142,14 @@ def partition(n, nranks, rank):
     return nl.value, off.value
 
 
-def validate(lattice, nx, ny, nz, tau, regularization="projective", boundary=None, nranks=1):
+def validate(lattice, nx, ny, nz, tau, regularization="projective", boundary=None, nranks=1,
+             representation="moments"):
     """Status mrlbm_create would return for these arguments (no GPU needed)."""
     keep = []
     D = 2 if lattice == "D2Q9" else 3
     b = make_boundary(boundary, D, keep)
-    return lib.mrlbm_validate(LATTICES[lattice], nx, ny, nz if D == 3 else 1, float(tau), REGS[regularization],
-                              ctypes.byref(b), nranks)
+    return lib.mrlbm_validate_repr(LATTICES[lattice], nx, ny, nz if D == 3 else 1, float(tau), REGS[regularization],
+                                   ctypes.byref(b), nranks, REPRS[representation])
 
 
 def step_group(solvers, n):
@@ -162,8 +168,10 @@ class Solver:
     """One mrlbm_t handle (see include/mrlbm.h for the semantics)."""
 
     def __init__(self, lattice, nx, ny, nz=1, tau=0.6, regularization="projective", boundary=None,
-                 precision="fp64", device=-1, stream=None, rank=0, nranks=1, nccl_id: bytes | None = None):
+                 precision="fp64", device=-1, stream=None, rank=0, nranks=1, nccl_id: bytes | None = None,
+                 representation="moments"):
         self.lattice, self.regularization, self.precision = lattice, regularization, precision
+        self.representation = representation
         self.D = 2 if lattice == "D2Q9" else 3
         self.M, self.Q = M_OF[lattice], Q_OF[lattice]
         self.nx, self.ny, self.nz = nx, ny, (nz if self.D == 3 else 1)
@@ -175,6 +183,7 @@ class Solver:
         o.device = device
         o.cuda_stream = stream
         o.rank, o.nranks = rank, nranks
+        o.representation = REPRS[representation]
         if nccl_id is not None:
             self._id = ctypes.create_string_buffer(bytes(nccl_id), 128)
             o.nccl_unique_id = ctypes.cast(self._id, ctypes.c_void_p)
@@ -221,6 +230,13 @@ class Solver:
         _check(lib.mrlbm_get_populations(self._h, out.ctypes.data_as(ctypes.POINTER(ctypes.c_double)), out.size),
                "mrlbm_get_populations")
         return out
+
+    def set_populations(self, f):
+        """pre-collision populations [Q][...] (fp64): stored as is (distributions)
+        or as their moments (moments representation)."""
+        a = np.ascontiguousarray(f, dtype=np.float64)
+        _check(lib.mrlbm_set_populations(self._h, a.ctypes.data_as(ctypes.POINTER(ctypes.c_double)), a.size),
+               "mrlbm_set_populations")
 
     # ---- device I/O (torch fp64 CUDA tensors in the ABI layout)
     def set_moments_device(self, t):

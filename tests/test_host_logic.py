@@ -34,6 +34,8 @@ def test_library_is_built_for_sm100a():
     sass = subprocess.run(["cuobjdump", "-sass", str(mrlbm._LIB_PATH)], capture_output=True, text=True).stdout
     # the fused step kernels stage their tiles with TMA (UTMALDG) and mbarriers (SYNCS)
     assert "mrlbm_step_kernel" in sass and "UTMALDG" in sass and "SYNCS" in sass
+    # the distribution-representation (ST) baseline kernels are in the same library
+    assert "st_step_kernel" in sass
 
 
 def test_status_strings():
@@ -79,6 +81,24 @@ def test_validation_codes():
     b["x+"] = {"kind": "pressure", "rho": 1.0}
     assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, boundary=b) == 0
     assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, nranks=8) == INV  # < 2 layers per rank
+
+
+def test_validation_codes_distribution_representation():
+    INV, UNS = -1, -2
+    # BGK (Alg. 1) is not moment-closed: distributions only
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, "bgk") == UNS
+    for reg in ("bgk", "projective", "recursive"):
+        assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, reg, representation="distributions") == 0
+    b = walls(3)
+    b["y+"] = {"kind": "moving_wall", "u": [0.1, 0.0, 0.0]}
+    assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, "bgk", boundary=walls(2), representation="distributions") == 0
+    assert mrlbm.validate("D3Q27", 8, 8, 8, 0.6, "bgk", boundary=b, representation="distributions") == 0
+    b = walls(2)
+    b["x-"] = {"kind": "velocity", "u": [0.01, 0, 0]}
+    b["x+"] = {"kind": "pressure", "rho": 1.0}
+    assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, boundary=b, representation="distributions") == UNS
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, nranks=2, representation="distributions") == UNS
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.5, "bgk", representation="distributions") == INV
 
 
 def test_create_fails_loudly_without_gpu():
