@@ -634,11 +634,18 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         }
     }
 
-    Real acc[3][M]; // rolling accumulators for layers c-1, c, c+1
+    // Two accumulator sets suffice for the three layers an arrival can reach
+    // (c-1, c, c+1): layer c-1 is completed and stored by the c_m = -1 group
+    // before anything is added to layer c+1, whose sums then reuse its
+    // registers.  The roles of the two sets alternate from layer to layer
+    // (the sweep is unrolled by two), so no accumulator is ever moved.
+    Real accA[M], accB[M], accC[M];
 #pragma unroll
-    for (int j = 0; j < 3; j++)
-#pragma unroll
-        for (int q = 0; q < M; q++) acc[j][q] = Real(0);
+    for (int q = 0; q < M; q++) {
+        accA[q] = Real(0);
+        accB[q] = Real(0);
+        accC[q] = Real(0);
+    }
 
     // ---- finalize the completed layer and store it (eqs 1-3; open faces R14)
     Real *const dst_node = dst + (long long)b * p.pitch + a; // this thread's node in plane 0
@@ -679,8 +686,11 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         }
     };
 
-    // one layer of the sweep with accumulators X (layer c-1), Y (c), Z (c+1)
-    auto layer = [&](const int it, Real (&X)[M], Real (&Y)[M], Real (&Z)[M]) {
+    // one layer of the sweep: on entry X holds layer c-1 and Y layer c; on
+    // exit Y holds layer c and Z layer c+1.  Z is X (ALIAS, two-set scheme)
+    // or a third, zeroed set (rotation scheme)
+    auto layer = [&](const int it, Real (&X)[M], Real (&Y)[M], Real (&Z)[M], auto alias_tag) {
+        constexpr bool ALIAS = decltype(alias_tag)::value;
         const int c = cfirst + it;
         const int s = it % S;
         mbar_wait(&full[s], (it / S) & 1);
@@ -753,6 +763,10 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                 };
                 pull(std::integral_constant<int, -1>{});
                 if (c - 1 >= c0 && c - 1 < c1) finalize_store(X, c - 1);
+                if constexpr (ALIAS) {
+#pragma unroll
+                    for (int q = 0; q < M; q++) X[q] = Real(0); // X becomes layer c+1
+                }
                 pull(std::integral_constant<int, 0>{});
                 pull(std::integral_constant<int, 1>{});
                 // halfway bounce-back at walls (R12, R13), out of line
@@ -768,44 +782,30 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
             else body(std::false_type{});
         }
     };
-    auto zero = [&](Real (&X)[M]) {
-#pragma unroll
-        for (int q = 0; q < M; q++) X[q] = Real(0);
-    };
-    if constexpr (D == 2 && sizeof(Real) == 4) {
-        // unrolled by 3: the accumulator roles rotate by renaming, not by moves
-        // (measured: +29% on C2 fp32; slower for fp64, whose unrolled body spills,
-        // and 5x slower for the 3D bodies, which then overflow the instruction cache)
-        for (int it = 0; it < nl; it += 3) {
-            layer(it, acc[0], acc[1], acc[2]);
-            zero(acc[0]);
-            if (it + 1 < nl) {
-                layer(it + 1, acc[1], acc[2], acc[0]);
-                zero(acc[1]);
-            }
-            if (it + 2 < nl) {
-                layer(it + 2, acc[2], acc[0], acc[1]);
-                zero(acc[2]);
-            }
+    if constexpr (!(LAT == LAT_D3Q27 && REC)) {
+        for (int it = 0; it < nl; it += 2) {
+            layer(it, accA, accB, accA, std::true_type{});
+            if (it + 1 < nl) layer(it + 1, accB, accA, accB, std::true_type{});
         }
+        // the last layer of the segment, when no halo layer follows it, is
+        // complete after the sweep: it is the Y of the last layer call
         if (owner && clast == c1 - 1) {
-            const int y = nl % 3; // the Y of the last layer call
-            if (y == 0) finalize_store(acc[0], c1 - 1);
-            else if (y == 1) finalize_store(acc[1], c1 - 1);
-            else finalize_store(acc[2], c1 - 1);
+            if (nl & 1) finalize_store(accB, c1 - 1);
+            else finalize_store(accA, c1 - 1);
         }
     } else {
+        // D3Q27 recursive: the body unrolled twice no longer fits the register
+        // file (local-memory spills), so one body and three rotating sets
         for (int it = 0; it < nl; it++) {
-            layer(it, acc[0], acc[1], acc[2]);
-            // rotate the accumulator window
+            layer(it, accA, accB, accC, std::false_type{});
 #pragma unroll
             for (int q = 0; q < M; q++) {
-                acc[0][q] = acc[1][q];
-                acc[1][q] = acc[2][q];
-                acc[2][q] = Real(0);
+                accA[q] = accB[q];
+                accB[q] = accC[q];
+                accC[q] = Real(0);
             }
         }
-        if (owner && clast == c1 - 1) finalize_store(acc[0], c1 - 1);
+        if (owner && clast == c1 - 1) finalize_store(accA, c1 - 1);
     }
 }
 
