@@ -540,6 +540,12 @@ __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> finalize_open(RVec<Real, 
 }
 
 // ------------------------------------------------------------ step kernel
+// Accumulator scheme of the sweep (see the kernel): two sets with alternating
+// roles, except D3Q27 recursive, whose body unrolled twice spills registers
+template <int LAT, bool REC> struct Sweep {
+    static constexpr bool two_set = !(LAT == LAT_D3Q27 && REC);
+};
+
 template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
     using L = Lattice<LAT>;
     static constexpr int NT = TA * TB;
@@ -689,8 +695,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     // one layer of the sweep: on entry X holds layer c-1 and Y layer c; on
     // exit Y holds layer c and Z layer c+1.  Z is X (ALIAS, two-set scheme)
     // or a third, zeroed set (rotation scheme)
-    auto layer = [&](const int it, Real (&X)[M], Real (&Y)[M], Real (&Z)[M], auto alias_tag) {
-        constexpr bool ALIAS = decltype(alias_tag)::value;
+    auto layer = [&](const int it, Real (&X)[M], Real (&Y)[M], Real (&Z)[M]) {
         const int c = cfirst + it;
         const int s = it % S;
         mbar_wait(&full[s], (it / S) & 1);
@@ -763,7 +768,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                 };
                 pull(std::integral_constant<int, -1>{});
                 if (c - 1 >= c0 && c - 1 < c1) finalize_store(X, c - 1);
-                if constexpr (ALIAS) {
+                if constexpr (Sweep<LAT, REC>::two_set) {
 #pragma unroll
                     for (int q = 0; q < M; q++) X[q] = Real(0); // X becomes layer c+1
                 }
@@ -782,10 +787,10 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
             else body(std::false_type{});
         }
     };
-    if constexpr (!(LAT == LAT_D3Q27 && REC)) {
+    if constexpr (Sweep<LAT, REC>::two_set) {
         for (int it = 0; it < nl; it += 2) {
-            layer(it, accA, accB, accA, std::true_type{});
-            if (it + 1 < nl) layer(it + 1, accB, accA, accB, std::true_type{});
+            layer(it, accA, accB, accA);
+            if (it + 1 < nl) layer(it + 1, accB, accA, accB);
         }
         // the last layer of the segment, when no halo layer follows it, is
         // complete after the sweep: it is the Y of the last layer call
@@ -797,7 +802,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         // D3Q27 recursive: the body unrolled twice no longer fits the register
         // file (local-memory spills), so one body and three rotating sets
         for (int it = 0; it < nl; it++) {
-            layer(it, accA, accB, accC, std::false_type{});
+            layer(it, accA, accB, accC);
 #pragma unroll
             for (int q = 0; q < M; q++) {
                 accA[q] = accB[q];
