@@ -142,6 +142,16 @@ template <class L> struct Axes {
         return s;
     }
     static constexpr int NMOVE = slot(L::Q);
+    // movers along B (c_b != 0): the ones that cross warps when a warp holds one
+    // A-row of the tile (3D kernels); the others move along A only
+    static constexpr bool bmover(int i) { return cb(i) != 0; }
+    static constexpr int bslot(int i)
+    {
+        int s = 0;
+        for (int k = 0; k < i; k++) s += bmover(k) ? 1 : 0;
+        return s;
+    }
+    static constexpr int NBMOVE = bslot(L::Q);
     static constexpr int opp(int i) { return i == 0 ? 0 : (i <= L::HALF ? i + L::HALF : i - L::HALF); }
 };
 

@@ -111,8 +111,11 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile)
         // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
         constexpr bool small_only = LAT == mr::LAT_D3Q27 && f64;
         if (tile == 0) tile = (LAT == mr::LAT_D3Q19 || small_only) ? 1 : 2;
-        if (tile == 1 || small_only) return make_variant<LAT, REC, Real, 32, 8, (f64 ? 2 : 3), 2>();
-        return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 3), 1>();
+        // TMA ring depth: with the A-movers exchanged by shuffles the fp64 32x8
+        // tile fits three stages at two CTAs per SM; the 32x16 tile (one CTA
+        // per SM) takes four in fp32
+        if (tile == 1 || small_only) return make_variant<LAT, REC, Real, 32, 8, 3, 2>();
+        return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 4), 1>();
     }
 }
 

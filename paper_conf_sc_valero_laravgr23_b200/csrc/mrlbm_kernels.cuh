@@ -430,12 +430,13 @@ __device__ __forceinline__ float rcp_nr(float x)
 
 // Halfway bounce-back (push form at the emitting node, R12) with the moving-wall
 // term (R13): the raw-moment increment of the node's own layer.  fl = this
-// thread's slot in the exchange plane (stride NT), fzm / fzp = its non-moving
-// populations with c_m = -1 / +1; wt weights arrivals on an open face (R14).
-template <int LAT, typename Real, int NT>
-__device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *fl, Real fzm, Real fzp, int bbA, int bbB,
-                                                              int bbC, Real rho_own, const StepArgs *p, int nx_in,
-                                                              int ny_in, bool open)
+// thread's slot in the exchange plane (stride NT), holding the movers that
+// went through shared memory (SHFL: only those with c_b != 0); the others are
+// read from fown; wt weights arrivals on an open face (R14).
+template <int LAT, typename Real, int NT, bool SHFL>
+__device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *fl, const Real (&fown)[Lattice<LAT>::Q],
+                                                              int bbA, int bbB, int bbC, Real rho_own,
+                                                              const StepArgs *p, int nx_in, int ny_in, bool open)
 {
     using L = Lattice<LAT>;
     using X = Axes<L>;
@@ -450,8 +451,9 @@ __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *f
         const bool xC = (cm != 0) && (cm == bbC);
         if (xA || xB || xC) {
             Real v;
-            if constexpr (X::moving(k)) v = fl[X::slot(k) * NT];
-            else v = (cm < 0) ? fzm : fzp;
+            if constexpr (SHFL && X::bmover(k)) v = fl[X::bslot(k) * NT];
+            else if constexpr (!SHFL && X::moving(k)) v = fl[X::slot(k) * NT];
+            else v = fown[k];
             constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
             constexpr double wk6 = 6.0 * L::w[k];
             double cuw = 0.0;
@@ -546,16 +548,28 @@ template <int LAT, bool REC> struct Sweep {
     static constexpr bool two_set = !(LAT == LAT_D3Q27 && REC);
 };
 
+// exchange-plane slot of population k, or -1 if it does not go through shared
+// memory (SHFL: only the c_b != 0 movers do; the others are shuffled or stay)
+template <class L, bool SHFL> constexpr int xslot_of(int k)
+{
+    if (SHFL) return Axes<L>::bmover(k) ? Axes<L>::bslot(k) : -1;
+    return Axes<L>::moving(k) ? Axes<L>::slot(k) : -1;
+}
+
 template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
     using L = Lattice<LAT>;
     static constexpr int NT = TA * TB;
+    // 3D tiles one warp wide: populations moving only along A are exchanged
+    // with warp shuffles, only the c_b != 0 movers go through shared memory
+    static constexpr bool SHFL = L::D == 3 && TA == 32;
+    static constexpr int NX = SHFL ? Axes<L>::NBMOVE : Axes<L>::NMOVE; // movers in the exchange plane
     // TMA box rows must start on a 16-byte boundary: the box starts at the
     // window origin rounded down to AL elements and is BW elements wide.
     static constexpr int AL = 16 / int(sizeof(Real));
     static constexpr int BW = (TA + AL - 1 + AL - 1) / AL * AL;
     static constexpr size_t box_elems = size_t(L::M) * TB * BW;
     static constexpr size_t stage_elems = (box_elems * sizeof(Real) + 127) / 128 * 128 / sizeof(Real);
-    static constexpr size_t F_elems = size_t(Axes<L>::NMOVE) * NT; // one exchange plane
+    static constexpr size_t F_elems = size_t(NX) * NT; // one exchange plane
     // two exchange planes (alternating layers) -> one __syncthreads per layer
     static constexpr size_t bytes = (S * stage_elems + 2 * F_elems) * sizeof(Real) + S * sizeof(uint64_t) + 128;
 };
@@ -570,6 +584,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     constexpr int HB = (D == 3) ? 1 : 0; // halo rows along B
     constexpr int NT = TA * TB;
     using SM = StepSmem<LAT, Real, TA, TB, S>;
+    constexpr bool SHFL = SM::SHFL;
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
     Real *stage = reinterpret_cast<Real *>(smem_raw);
@@ -602,6 +617,15 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     const bool valid = (inA || (perA && (a == -1 || a == nA))) && (inB || (perB && (b == -1 || b == nB)));
     const bool interior = tx >= 1 && tx < TA - 1 && ty >= HB && ty < TB - HB;
     const bool owner = interior && inA && inB;
+    // SHFL: every lane of an interior row runs the streaming code (a warp is one
+    // row, so the shuffles see all 32 lanes); only owners store
+    const bool stream_lane = SHFL ? (ty >= HB && ty < TB - HB) : owner;
+    // open faces in this CTA's window (CTA-uniform, so that the weighted and the
+    // plain streaming bodies never diverge inside a warp)
+    const int tilesB_ = gridDim.x / p.tilesA;
+    const bool cta_open = (p.kind[0] >= BC_VELOCITY && tA == 0) || (p.kind[1] >= BC_VELOCITY && tA == p.tilesA - 1) ||
+                          (D == 3 && ((p.kind[2] >= BC_VELOCITY && tB == 0) ||
+                                      (p.kind[3] >= BC_VELOCITY && tB == tilesB_ - 1)));
     // ghost shift of an owner on a periodic edge: a = 0 -> column nA, a = nA-1 -> column -1
     const int gA = !perA ? 0 : (a == 0 ? nA : (a == nA - 1 ? -nA : 0));
     const int gB = (D == 2 || !perB) ? 0 : (b == 0 ? nB : (b == nB - 1 ? -nB : 0));
@@ -676,6 +700,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
 #pragma unroll
             for (int q = 0; q < M; q++) out[q] = ov.v[q];
         }
+        if (!owner) return;
         Real *o = dst_node + (long long)(c + 1) * p.pstride;
 #pragma unroll
         for (int q = 0; q < M; q++) o[q * p.mstride] = out[q];
@@ -719,12 +744,14 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
             reconstruct<LAT, REC, Real>(A, fown);
             rho_own = Real(1) + m[0];
             static_for<0, Q>([&](auto kk) {
-                constexpr int k = decltype(kk)::value;
-                if constexpr (X::moving(k)) Fl[X::slot(k) * NT + tid] = fown[k];
+                constexpr int xs = xslot_of<L, SM::SHFL>(decltype(kk)::value);
+                if constexpr (xs >= 0) Fl[xs * NT + tid] = fown[decltype(kk)::value];
             });
         } else {
 #pragma unroll
-            for (int q = 0; q < X::NMOVE; q++) Fl[q * NT + tid] = Real(0);
+            for (int q = 0; q < SM::NX; q++) Fl[q * NT + tid] = Real(0);
+#pragma unroll
+            for (int q = 0; q < Q; q++) fown[q] = Real(0);
         }
         // one barrier per layer: the other exchange plane was last read before
         // this barrier, and every thread has read stage s
@@ -734,7 +761,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
             tma_load_4d(stage + s * SM::stage_elems, &tmap, &full[s], boxA, b0 + p.padB, 0, plane_of(c + S));
         }
 
-        if (owner) {
+        if (stream_lane) {
             const int bbC = (c == 0 && !p.lo_nb) ? -1 : ((c == nC - 1 && !p.hi_nb) ? 1 : 0);
             auto body = [&](auto open_tag) {
                 constexpr bool OPEN = decltype(open_tag)::value;
@@ -755,7 +782,9 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                             return OV<false, Real>{};
                         } else {
                             Real v;
-                            if constexpr (X::moving(k)) v = Fl[X::slot(k) * NT + (ty - cb) * TA + (tx - ca)];
+                            constexpr int xs = xslot_of<L, SM::SHFL>(k);
+                            if constexpr (xs >= 0) v = Fl[xs * NT + (ty - cb) * TA + (tx - ca)];
+                            else if constexpr (ca != 0) v = __shfl_sync(0xffffffffu, fown[k], tx - ca);
                             else v = fown[k];
                             if constexpr (OPEN) {
                                 constexpr int kx = L::c[k][0], ky = L::c[k][1];
@@ -776,14 +805,13 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                 pull(std::integral_constant<int, 1>{});
                 // halfway bounce-back at walls (R12, R13), out of line
                 if (bbA | bbB | bbC) {
-                    constexpr int kzm = dir_of<L>(0, 0, -1), kzp = dir_of<L>(0, 0, 1);
-                    const RVec<Real, M> d = bounce_back<LAT, Real, NT>(Fl + tid, fown[kzm], fown[kzp], bbA, bbB, bbC,
-                                                                       rho_own, &p, nx_in, ny_in, OPEN);
+                    const RVec<Real, M> d = bounce_back<LAT, Real, NT, SM::SHFL>(Fl + tid, fown, bbA, bbB, bbC, rho_own, &p,
+                                                                             nx_in, ny_in, OPEN);
 #pragma unroll
                     for (int q = 0; q < M; q++) Y[q] += d.v[q];
                 }
             };
-            if (openF >= 0) body(std::true_type{});
+            if (SM::SHFL ? cta_open : openF >= 0) body(std::true_type{});
             else body(std::false_type{});
         }
     };
