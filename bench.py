@@ -56,6 +56,12 @@ def load_peaks():
 
 
 def build_config(name, precision, n_ranks):
+    if name == "C5":
+        # C5w: one 1024 x 1024 x 128 slab per GPU of the 1024^3 channel
+        # (the full 1024^3 fp64 state, 172 GB in two copies, is the P = 8 weak point)
+        c = configs.c5(nz=128 * n_ranks)
+        c.precision = precision
+        return c
     c = configs.ALL[name]() if name != "C2" else configs.c2(precision)
     c.precision = precision
     if n_ranks > 1:
@@ -190,7 +196,7 @@ def workload_config(c, world):
     dims = f"{c.nx}x{c.ny}" if c.D == 2 else f"{c.nx}x{c.ny}x{c.nz}"
     coll = "BGK" if c.regularization == "bgk" else f"{c.regularization}-regularized"
     return {"workload": f"{c.name}: {c.lattice} {coll} "
-                        f"{'lid-driven cavity' if 'y+' in c.boundary and c.boundary['y+']['kind'] == 'moving_wall' else 'flow'} "
+                        f"{'lid-driven cavity' if 'y+' in c.boundary and c.boundary['y+']['kind'] == 'moving_wall' else ('channel' if c.name == 'C5' else 'flow')} "
                         f"{dims} {c.precision}",
             "lattice": c.lattice, "regularization": c.regularization, "grid": dims, "tau": c.tau,
             "precision": c.precision, "nodes": c.nodes,

@@ -42,16 +42,18 @@ def needs_build() -> bool:
     return any(p.stat().st_mtime > t for p in DEPS)
 
 
-def build(force: bool = False, verbose: bool = False) -> Path:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, out: Path | None = None, defines=()) -> Path:
+    """out / defines: a variant build for A/B comparisons (e.g. ab/libmrlbm_X.so, -DNAME)."""
+    target = Path(out) if out else LIB
+    if not force and not out and not needs_build():
         return LIB
     inc, lib = nccl_dirs()
     ncclso = "libnccl.so.2" if (lib / "libnccl.so.2").exists() else "libnccl.so"
-    tmp = LIB.with_suffix(f".{os.getpid()}.tmp.so")
+    tmp = target.with_suffix(f".{os.getpid()}.tmp.so")
     cmd = [nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "--expt-relaxed-constexpr",
            "-Xcompiler", "-fPIC", "-shared", "-o", str(tmp), *map(str, SOURCES),
            f"-I{ROOT / 'include'}", f"-I{inc}", f"-L{lib}", f"-l:{ncclso}",
-           "-Xlinker", f"-rpath,{lib}"]
+           "-Xlinker", f"-rpath,{lib}", *[f"-D{d}" for d in defines]]
     if verbose:
         cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -60,10 +62,12 @@ def build(force: bool = False, verbose: bool = False) -> Path:
         raise RuntimeError("nvcc failed building libmrlbm.so")
     if verbose:
         sys.stderr.write(r.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose="-v" in sys.argv)
-    print(LIB)
+    a = sys.argv[1:]
+    out = a[a.index("-o") + 1] if "-o" in a else None
+    defs = [x[2:] for x in a if x.startswith("-D")]
+    print(build(force="--force" in a, verbose="-v" in a, out=out, defines=defs))

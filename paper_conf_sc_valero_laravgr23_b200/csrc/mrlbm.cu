@@ -104,7 +104,10 @@ template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB> Var
 template <int LAT, bool REC, typename Real> Variant pick(int tile)
 {
     if constexpr (LAT == mr::LAT_D2Q9) {
+        // deeper TMA rings trade resident CTAs for bytes in flight (tuning: MRLBM_TILE)
         if (tile == 1) return make_variant<LAT, REC, Real, 128, 1, 4, 4>();
+        if (tile == 2) return make_variant<LAT, REC, Real, 128, 1, 6, 4>();
+        if (tile == 3) return make_variant<LAT, REC, Real, 128, 1, 8, 3>();
         return make_variant<LAT, REC, Real, 128, 1, 4, 5>();
     } else {
         constexpr bool f64 = sizeof(Real) == 8;

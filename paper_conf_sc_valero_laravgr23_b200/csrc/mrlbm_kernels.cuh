@@ -108,8 +108,14 @@ __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map)
 // C(h_a, 2) times and (a,b), a < b, h_a h_b times, so every term is one FMA
 // against a monomial u^m (m <= (2,2,2)) computed once per node.
 // The full tensor bases (D2Q9 / D3Q27 recursive) use the sum-factorised
-// reconstruction, which applies the per-axis Hermite scale itself.
+// reconstruction, which applies the per-axis Hermite scale and the D1Q3
+// weights itself; their coefficients carry only tscale(h) = 6^-(#axes with h = 0).
 template <int LAT, bool REC> constexpr bool tensor_recon() { return REC && LAT != LAT_D3Q19; }
+constexpr double tscale(int D, int h0, int h1, int h2)
+{
+    const int z = (h0 == 0) + (h1 == 0) + (D == 3 && h2 == 0);
+    return z == 0 ? 1.0 : (z == 1 ? 1.0 / 6 : (z == 2 ? 1.0 / 36 : 1.0 / 216));
+}
 
 template <int LAT, bool REC, typename Real>
 __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M], Real omega,
@@ -159,16 +165,21 @@ __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M],
         constexpr int k = decltype(hk)::value;
         constexpr int h0 = B::h[k][0], h1 = B::h[k][1], h2 = B::h[k][2];
         constexpr int n = h0 + h1 + h2;
+        constexpr bool TS = tensor_recon<LAT, REC>();
         constexpr Real sc = Real(hscale(h0, h1, h2));
+        // tensor bases: the weight scale rides on rho and omega (one product per
+        // distinct scale, shared by every component that has it)
+        constexpr Real ts = Real(TS ? tscale(D, h0, h1, h2) : 1.0);
         constexpr int i0 = (h0 > 0) ? 0 : ((h1 > 0) ? 1 : 2);
         Real val;
         if constexpr (n == 0) {
-            val = drho;
+            val = TS ? drho * ts : drho;
         } else if constexpr (n == 1) {
-            val = rho * u[i0];
+            val = (TS ? rho * ts : rho) * u[i0];
         } else if constexpr (n == 2) {
             constexpr int i1 = (h0 == 2) ? 0 : ((h0 == 1) ? ((h1 > 0) ? 1 : 2) : ((h1 == 2) ? 1 : 2));
-            val = omega * m[pslot<D>(i0, i1)] + omc * rho * u[i0] * u[i1];
+            if constexpr (TS) val = fma(omega * ts, m[pslot<D>(i0, i1)], (omc * rho * ts) * (u[i0] * u[i1]));
+            else val = omega * m[pslot<D>(i0, i1)] + omc * rho * u[i0] * u[i1];
         } else {
             using H0 = std::integral_constant<int, h0>;
             using H1 = std::integral_constant<int, h1>;
@@ -188,9 +199,10 @@ __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M],
             if constexpr (h1 * h2 > 0)
                 aneq = fma(Real(h1 * h2) * Pn[1][2],
                            mono(H0{}, std::integral_constant<int, h1 - 1>{}, std::integral_constant<int, h2 - 1>{}), aneq);
-            val = fma(omega, aneq, rho * mono(H0{}, H1{}, H2{}));
+            if constexpr (TS) val = fma(omega * ts, aneq, (rho * ts) * mono(H0{}, H1{}, H2{}));
+            else val = fma(omega, aneq, rho * mono(H0{}, H1{}, H2{}));
         }
-        if constexpr (tensor_recon<LAT, REC>()) A[k] = val; // scale folded into synth3
+        if constexpr (TS) A[k] = val; // Hermite scale and weights folded into synth3w
         else A[k] = val * sc;
     });
 }
@@ -202,21 +214,23 @@ template <int LAT, bool REC> constexpr int hindex(int a, int b, int c)
     return -1;
 }
 
-// 1D Hermite synthesis at c = -1, 0, +1 with the per-axis scale folded in:
-// hscale(a,b,c) = s(a) s(b) s(c), s(0) = 1, s(1) = 3, s(2) = 3/2, so
-//   g(c) = A0 + 3 c A1 + (3/2)(3c^2 - 1) A2:  g(0) = A0 - 3/2 A2,  g(+-1) = A0 + 3 A2 +- 3 A1
+// Weighted 1D Hermite synthesis at c = -1, 0, +1: the per-axis Hermite scale
+// hscale(a,b,c) = s(a) s(b) s(c) (s(0) = 1, s(1) = 3, s(2) = 3/2) and the D1Q3
+// weight w(0) = 2/3, w(+-1) = 1/6 folded in, for a0 = A0 / 6 (tscale):
+//   G(0) = w(0) (A0 - 3/2 A2) = 4 a0 - A2,  G(+-1) = w(1) (A0 + 3 A2 +- 3 A1) = a0 + A2/2 +- A1/2
 template <typename Real>
-__device__ __forceinline__ void synth3(Real A0, Real A1, Real A2, Real &gm, Real &g0, Real &gp)
+__device__ __forceinline__ void synth3w(Real a0, Real A1, Real A2, Real &gm, Real &g0, Real &gp)
 {
-    const Real S = fma(Real(3), A2, A0);
-    g0 = fma(Real(-1.5), A2, A0);
-    gp = fma(Real(3), A1, S);
-    gm = fma(Real(-3), A1, S);
+    const Real S = fma(Real(0.5), A2, a0);
+    g0 = fma(Real(4), a0, -A2);
+    gp = fma(Real(0.5), A1, S);
+    gm = fma(Real(-0.5), A1, S);
 }
 
 // Sum-factorised eq 14 for the full tensor bases {0,1,2}^D (D2Q9 / D3Q27
-// recursive): the Hermite-to-population map is the D-fold tensor product of
-// the 1D map above, applied axis by axis (z, y, x), then times w_i.
+// recursive): the Hermite-to-population map times w_i is the D-fold tensor
+// product of the weighted 1D map above (the weights are D1Q3 products),
+// applied axis by axis (z, y, x).  Coefficients arrive scaled by tscale(h).
 template <int LAT, typename Real>
 __device__ __forceinline__ void reconstruct_tensor(const Real (&A)[Basis<LAT, true>::NH], Real (&f)[Lattice<LAT>::Q])
 {
@@ -230,7 +244,7 @@ __device__ __forceinline__ void reconstruct_tensor(const Real (&A)[Basis<LAT, tr
         if constexpr (D == 3) {
             constexpr int k1 = hindex<LAT, true>(a, b, 1), k2 = hindex<LAT, true>(a, b, 2);
             static_assert(k1 >= 0 && k2 >= 0, "basis component missing");
-            synth3(A[k0], A[k1], A[k2], T[a][b][0], T[a][b][1], T[a][b][2]);
+            synth3w(A[k0], A[k1], A[k2], T[a][b][0], T[a][b][1], T[a][b][2]);
         } else {
             T[a][b][1] = A[k0];
         }
@@ -240,17 +254,16 @@ __device__ __forceinline__ void reconstruct_tensor(const Real (&A)[Basis<LAT, tr
 #pragma unroll
     for (int a = 0; a < 3; a++)
 #pragma unroll
-        for (int zi = z0; zi < z1; zi++) synth3(T[a][0][zi], T[a][1][zi], T[a][2][zi], U[a][0][zi], U[a][1][zi], U[a][2][zi]);
+        for (int zi = z0; zi < z1; zi++) synth3w(T[a][0][zi], T[a][1][zi], T[a][2][zi], U[a][0][zi], U[a][1][zi], U[a][2][zi]);
     Real V[3][3][3]; // [c_x + 1][c_y + 1][c_z + 1]
 #pragma unroll
     for (int yi = 0; yi < 3; yi++)
 #pragma unroll
-        for (int zi = z0; zi < z1; zi++) synth3(U[0][yi][zi], U[1][yi][zi], U[2][yi][zi], V[0][yi][zi], V[1][yi][zi], V[2][yi][zi]);
+        for (int zi = z0; zi < z1; zi++) synth3w(U[0][yi][zi], U[1][yi][zi], U[2][yi][zi], V[0][yi][zi], V[1][yi][zi], V[2][yi][zi]);
     static_for<0, L::Q>([&](auto ik) {
         constexpr int i = decltype(ik)::value;
-        constexpr Real w = Real(L::w[i]);
         constexpr int xi = L::c[i][0] + 1, yi = L::c[i][1] + 1, zi = L::c[i][2] + 1;
-        f[i] = w * V[xi][yi][zi];
+        f[i] = V[xi][yi][zi];
     });
 }
 
@@ -332,11 +345,18 @@ template <bool A, bool B, typename Real> __device__ __forceinline__ auto ov_sub(
     else if constexpr (B) return OV<true, Real>{-b.v};
     else return OV<false, Real>{};
 }
-// acc += sgn * x  (sgn in {-1, 0, +1}, compile time)
-template <int SG, bool A, typename Real> __device__ __forceinline__ void ov_acc(Real &acc, OV<A, Real> x)
+// acc += sgn * x  (sgn in {-1, 0, +1}, compile time); ASSIGN: acc = sgn * x
+// (the first contribution to a fresh accumulator: no zeroing, no add)
+template <int SG, bool ASSIGN = false, bool A, typename Real> __device__ __forceinline__ void ov_acc(Real &acc, OV<A, Real> x)
 {
-    if constexpr (A && SG == 1) acc += x.v;
-    else if constexpr (A && SG == -1) acc -= x.v;
+    if constexpr (ASSIGN) {
+        if constexpr (A && SG == 1) acc = x.v;
+        else if constexpr (A && SG == -1) acc = -x.v;
+        else acc = Real(0);
+    } else {
+        if constexpr (A && SG == 1) acc += x.v;
+        else if constexpr (A && SG == -1) acc -= x.v;
+    }
 }
 template <class A, class B, class C> struct Tri {
     A r0;
@@ -363,7 +383,8 @@ template <class L> constexpr int dir_of(int ca, int cb, int cm)
 // Add the raw moments (sum f, sum c f, sum c c f) of the arrivals G(ia, ib)
 // that move by CM along the sweep axis to acc, sum-factorised: sums over c_a
 // per row c_b, then over c_b; the sweep component c_m = CM enters as a factor.
-template <class L, int CM, typename Real, class GF>
+// AS: acc is fresh (assigned, not added to).
+template <class L, int CM, bool AS, typename Real, class GF>
 __device__ __forceinline__ void accum_group(Real (&acc)[L::M], GF &&G)
 {
     constexpr int D = L::D;
@@ -382,22 +403,22 @@ __device__ __forceinline__ void accum_group(Real (&acc)[L::M], GF &&G)
     auto Saa = ov_add(ov_add(rp.r2, rm.r2), rz.r2);  // sum ca^2 f
     auto Sab = ov_sub(rp.r1, rm.r1);                 // sum ca cb f
     constexpr int CM2 = CM * CM;
-    ov_acc<1>(acc[0], S);
-    ov_acc<1>(acc[1], Sa);                           // j_x (A = x)
+    ov_acc<1, AS>(acc[0], S);
+    ov_acc<1, AS>(acc[1], Sa);                       // j_x (A = x)
     if constexpr (D == 3) {
-        ov_acc<1>(acc[2], Sb);                       // j_y (B = y)
-        ov_acc<CM>(acc[3], S);                       // j_z (C = z)
-        ov_acc<1>(acc[pslot<3>(0, 0)], Saa);
-        ov_acc<1>(acc[pslot<3>(1, 1)], Sbb);
-        ov_acc<CM2>(acc[pslot<3>(2, 2)], S);
-        ov_acc<1>(acc[pslot<3>(0, 1)], Sab);
-        ov_acc<CM>(acc[pslot<3>(0, 2)], Sa);
-        ov_acc<CM>(acc[pslot<3>(1, 2)], Sb);
+        ov_acc<1, AS>(acc[2], Sb);                   // j_y (B = y)
+        ov_acc<CM, AS>(acc[3], S);                   // j_z (C = z)
+        ov_acc<1, AS>(acc[pslot<3>(0, 0)], Saa);
+        ov_acc<1, AS>(acc[pslot<3>(1, 1)], Sbb);
+        ov_acc<CM2, AS>(acc[pslot<3>(2, 2)], S);
+        ov_acc<1, AS>(acc[pslot<3>(0, 1)], Sab);
+        ov_acc<CM, AS>(acc[pslot<3>(0, 2)], Sa);
+        ov_acc<CM, AS>(acc[pslot<3>(1, 2)], Sb);
     } else {                                         // 2D: C = y, no B axis
-        ov_acc<CM>(acc[2], S);
-        ov_acc<1>(acc[pslot<2>(0, 0)], Saa);
-        ov_acc<CM2>(acc[pslot<2>(1, 1)], S);
-        ov_acc<CM>(acc[pslot<2>(0, 1)], Sa);
+        ov_acc<CM, AS>(acc[2], S);
+        ov_acc<1, AS>(acc[pslot<2>(0, 0)], Saa);
+        ov_acc<CM2, AS>(acc[pslot<2>(1, 1)], S);
+        ov_acc<CM, AS>(acc[pslot<2>(0, 1)], Sa);
     }
 }
 
@@ -741,8 +762,8 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         if (valid) {
             Real A[Basis<LAT, REC>::NH];
             collide_coeffs<LAT, REC, Real>(m, omega, A);
-            reconstruct<LAT, REC, Real>(A, fown);
             rho_own = Real(1) + m[0];
+            reconstruct<LAT, REC, Real>(A, fown);
             static_for<0, Q>([&](auto kk) {
                 constexpr int xs = xslot_of<L, SM::SHFL>(decltype(kk)::value);
                 if constexpr (xs >= 0) Fl[xs * NT + tid] = fown[decltype(kk)::value];
@@ -793,16 +814,13 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                             return OV<true, Real>{v};
                         }
                     };
-                    accum_group<L, CM, Real>(CM < 0 ? X : (CM == 0 ? Y : Z), G);
+                    // the c_m = +1 group is the first contribution to layer c+1
+                    accum_group<L, CM, (CM > 0), Real>(CM < 0 ? X : (CM == 0 ? Y : Z), G);
                 };
                 pull(std::integral_constant<int, -1>{});
                 if (c - 1 >= c0 && c - 1 < c1) finalize_store(X, c - 1);
-                if constexpr (Sweep<LAT, REC>::two_set) {
-#pragma unroll
-                    for (int q = 0; q < M; q++) X[q] = Real(0); // X becomes layer c+1
-                }
                 pull(std::integral_constant<int, 0>{});
-                pull(std::integral_constant<int, 1>{});
+                pull(std::integral_constant<int, 1>{}); // assigns Z (= X in the two-set scheme)
                 // halfway bounce-back at walls (R12, R13), out of line
                 if (bbA | bbB | bbC) {
                     const RVec<Real, M> d = bounce_back<LAT, Real, NT, SM::SHFL>(Fl + tid, fown, bbA, bbB, bbC, rho_own, &p,
@@ -832,10 +850,9 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         for (int it = 0; it < nl; it++) {
             layer(it, accA, accB, accC);
 #pragma unroll
-            for (int q = 0; q < M; q++) {
+            for (int q = 0; q < M; q++) { // accC is assigned by the next layer's c_m = +1 group
                 accA[q] = accB[q];
                 accB[q] = accC[q];
-                accC[q] = Real(0);
             }
         }
         if (owner && clast == c1 - 1) finalize_store(accA, c1 - 1);

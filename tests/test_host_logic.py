@@ -114,3 +114,17 @@ def test_slab_cut_and_reassemble():
     m = np.random.default_rng(0).standard_normal((10, 13, 5, 4))
     parts = [distributed.slab_of(m, 4, r) for r in range(4)]
     assert np.array_equal(np.concatenate(parts, axis=1), m)
+
+
+def test_bench_workloads():
+    """bench.py's workloads: C2 is BASELINE configs[1]; C5 runs as the C5w slab
+    (1024 x 1024 x 128 per GPU) and grows along z with the ranks."""
+    import bench
+    c2 = bench.build_config("C2", "fp64", 1)
+    assert (c2.lattice, c2.regularization, c2.nx, c2.ny, c2.precision) == ("D2Q9", "recursive", 4096, 4096, "fp64")
+    assert bench.build_config("C2", "fp64", 4).ny == 4 * 4096
+    for world in (1, 2, 8):
+        c5 = bench.build_config("C5", "fp64", world)
+        assert (c5.lattice, c5.regularization, c5.nx, c5.ny, c5.nz) == ("D3Q19", "recursive", 1024, 1024, 128 * world)
+        assert c5.boundary["x-"]["u_profile"].shape == (128 * world, 1024, 3)
+    assert "channel" in bench.workload_config(bench.build_config("C5", "fp64", 1), 1)["workload"]

@@ -40,7 +40,11 @@ UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12
 
 
 def read_rep(path):
-    out = subprocess.run(["ncu", "-i", str(path), "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    """an .ncu-rep, or the `--page raw --csv` export of one (tools/ncu_capture.sh)"""
+    if str(path).endswith(".csv"):
+        out = Path(path).read_text()
+    else:
+        out = subprocess.run(["ncu", "-i", str(path), "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     hdr, units, vals = rows[0], rows[1], rows[2]
     res = {"kernel": vals[hdr.index("Kernel Name")] if "Kernel Name" in hdr else ""}
