@@ -24,7 +24,8 @@ _LIB = _HERE / "liboracle.so"
 
 LATTICES = {"D2Q9": 0, "D3Q19": 1, "D3Q27": 2}
 REGS = {"projective": 0, "recursive": 1, "bgk": 2}
-BC = {"periodic": 0, "wall": 1, "moving_wall": 2, "velocity": 3, "pressure": 4}
+BC = {"periodic": 0, "wall": 1, "moving_wall": 2, "velocity": 3, "pressure": 4,
+      "velocity_fd": 5, "pressure_fd": 6}
 FACES = ("x-", "x+", "y-", "y+", "z-", "z+")
 
 

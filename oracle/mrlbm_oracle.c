@@ -28,7 +28,9 @@
  *   walls             halfway bounce-back, link-wise (R12); moving wall
  *                     (Ladd), rho_w = node pre-collision rho (R13)
  *   open faces        regularized velocity / pressure (Latt et al. [6],
- *                     P:L283, R14)
+ *                     P:L283, R14); finite-difference variant (the scheme the
+ *                     paper's proxy apps used, "finite difference
+ *                     boundary conditions at the inlet and outlet [6]"; R20)
  *
  * Parity pins: every function here is pinned by tests/test_oracle_*.py against
  * lattice identities, closed forms (tau = 1, u = 0), the paper's eq 9 == eqs
@@ -49,7 +51,9 @@
 
 enum { D2Q9 = 0, D3Q19 = 1, D3Q27 = 2 };
 enum { PROJECTIVE = 0, RECURSIVE = 1, BGK = 2 };
-enum { PERIODIC = 0, WALL = 1, MOVING_WALL = 2, VELOCITY = 3, PRESSURE = 4 };
+enum { PERIODIC = 0, WALL = 1, MOVING_WALL = 2, VELOCITY = 3, PRESSURE = 4, VELOCITY_FD = 5, PRESSURE_FD = 6 };
+#define IS_OPEN(k) ((k) >= VELOCITY)
+#define IS_FD(k) ((k) >= VELOCITY_FD)
 
 typedef struct {
     int D, Q;
@@ -320,7 +324,7 @@ oracle_t *oracle_create(int lattice, int64_t nx, int64_t ny, int64_t nz, double 
         for (int a = 0; a < 3; a++) o->uw[F][a] = uw[3 * F + a];
         o->rhow[F] = rhow[F];
         if (o->L.D == 2 && F >= 4) o->kind[F] = PERIODIC;
-        if (uprof && uprof[F] && o->kind[F] == VELOCITY) {
+        if (uprof && uprof[F] && (o->kind[F] == VELOCITY || o->kind[F] == VELOCITY_FD)) {
             int ax = F / 2;
             int64_t cnt = o->N / o->n[ax] * o->L.D;
             o->uprof[F] = (double *)malloc(sizeof(double) * cnt);
@@ -448,7 +452,7 @@ static void open_face_node(oracle_t *o, int F, const int64_t p[3])
         if (cls[i] == -1) S += 2.0 * f[i];
     }
     double rho, u[3] = {0, 0, 0};
-    if (o->kind[F] == VELOCITY) {
+    if (o->kind[F] == VELOCITY || o->kind[F] == VELOCITY_FD) {
         if (o->uprof[F]) {
             int64_t fi = face_index(o, F, p);
             for (int a = 0; a < L->D; a++) u[a] = o->uprof[F][fi * L->D + a];
@@ -481,6 +485,76 @@ static void open_face_node(oracle_t *o, int F, const int64_t p[3])
             for (int b = 0; b < L->D; b++) HP += H2(L, i, a, b) * Pneq[a][b];
         o->fn[i * N + k] = feq[i] + L->w[i] / (2.0 * CS2 * CS2) * HP;
     }
+}
+
+/* Finite-difference open faces (Latt et al. [6], the "FD" scheme; R20).
+ * rho and u of a face node come from the same rule as the regularized face
+ * (open_face_node above: rho from the known populations on a velocity face,
+ * u.n from them on a pressure face).  The non-equilibrium part is the
+ * first-order Chapman-Enskog stress of the NEW velocity field,
+ *   Pi^neq_ab = -rho tau c_s^2 (d_a u_b + d_b u_a),
+ * with second-order finite differences: one-sided along the face normal,
+ *   d u = s (-3 u(0) + 4 u(s) - u(2s)) / 2   (s = inward direction),
+ * central along the face (wrapped on periodic axes), one-sided at the face's
+ * edges.  The node is then set to f = f^eq(rho, u) + w H2 : Pi^neq / (2 c_s^4),
+ * i.e. moments (rho, u, rho u u + Pi^neq). */
+static double fd_deriv(const oracle_t *o, const double *U, int ax, const int64_t p[3], int comp)
+{
+    const int64_t n = o->n[ax];
+    int64_t q[3] = {p[0], p[1], p[2]};
+    const int per = o->kind[2 * ax] == PERIODIC;
+    double um, u0, up;
+#define UAT(QQ) (U[3 * nid(o, (QQ)[0], (QQ)[1], (QQ)[2]) + comp])
+    if (per || (p[ax] > 0 && p[ax] < n - 1)) {
+        q[ax] = (p[ax] - 1 + n) % n; um = UAT(q);
+        q[ax] = (p[ax] + 1) % n; up = UAT(q);
+        return 0.5 * (up - um);
+    }
+    const int64_t s = (p[ax] == 0) ? 1 : -1;
+    u0 = UAT(p);
+    q[ax] = p[ax] + s; up = UAT(q);
+    q[ax] = p[ax] + 2 * s; um = UAT(q);
+#undef UAT
+    return (double)s * 0.5 * (-3.0 * u0 + 4.0 * up - um);
+}
+
+static void fd_faces(oracle_t *o)
+{
+    const lattice_t *L = &o->L;
+    const int64_t N = o->N;
+    double *U = (double *)malloc(sizeof(double) * 3 * N);
+    double *R = (double *)malloc(sizeof(double) * N);
+    for (int64_t k = 0; k < N; k++) {
+        double f[27];
+        for (int i = 0; i < L->Q; i++) f[i] = o->fn[i * N + k];
+        moments_of(L, f, &R[k], &U[3 * k], NULL);
+    }
+    for (int F = 0; F < 2 * L->D; F++) {
+        if (!IS_FD(o->kind[F])) continue;
+        int ax = F / 2;
+        int64_t fixed = (F % 2 == 0) ? 0 : o->n[ax] - 1;
+        for (int64_t k = 0; k < N; k++) {
+            int64_t p[3] = {k % o->n[0], (k / o->n[0]) % o->n[1], k / (o->n[0] * o->n[1])};
+            if (p[ax] != fixed) continue;
+            double g[3][3]; /* g[a][b] = d_a u_b */
+            memset(g, 0, sizeof(g));
+            for (int a = 0; a < L->D; a++)
+                for (int b = 0; b < L->D; b++) g[a][b] = fd_deriv(o, U, a, p, b);
+            const double rho = R[k];
+            double Pneq[3][3];
+            memset(Pneq, 0, sizeof(Pneq));
+            for (int a = 0; a < L->D; a++)
+                for (int b = 0; b < L->D; b++) Pneq[a][b] = -rho * o->tau * CS2 * (g[a][b] + g[b][a]);
+            for (int i = 0; i < L->Q; i++) {
+                double HP = 0;
+                for (int a = 0; a < L->D; a++)
+                    for (int b = 0; b < L->D; b++) HP += H2(L, i, a, b) * Pneq[a][b];
+                o->fn[i * N + k] = feq_i(L, i, rho, &U[3 * k]) + L->w[i] / (2.0 * CS2 * CS2) * HP;
+            }
+        }
+    }
+    free(U);
+    free(R);
 }
 
 static void stream_all(oracle_t *o)
@@ -522,8 +596,10 @@ static void stream_all(oracle_t *o)
         }
     }
     /* open faces after wall bounce-back (R14) */
+    int any_fd = 0;
     for (int F = 0; F < 2 * L->D; F++) {
-        if (o->kind[F] != VELOCITY && o->kind[F] != PRESSURE) continue;
+        if (!IS_OPEN(o->kind[F])) continue;
+        any_fd |= IS_FD(o->kind[F]);
         int ax = F / 2;
         int64_t fixed = (F % 2 == 0) ? 0 : o->n[ax] - 1;
         for (int64_t k = 0; k < N; k++) {
@@ -532,6 +608,7 @@ static void stream_all(oracle_t *o)
             open_face_node(o, F, p);
         }
     }
+    if (any_fd) fd_faces(o);
     double *t = o->f; o->f = o->fn; o->fn = t;
 }
 
