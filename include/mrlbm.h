@@ -75,18 +75,29 @@ typedef enum { MRLBM_FP64 = 0, MRLBM_FP32 = 1 } mrlbm_precision;
  *                rho = the node's pre-collision density; u_w tangential
  *   VELOCITY     regularized velocity face: u prescribed (u[] or u_profile)
  *   PRESSURE     regularized pressure face: rho prescribed, tangential u = 0
- * Open faces (VELOCITY/PRESSURE) are supported on the x and y faces of 3D
+ *   VELOCITY_FD, PRESSURE_FD
+ *                finite-difference faces of Latt et al. [6], the inlet /
+ *                outlet of the paper's proxy apps ("finite difference
+ *                boundary conditions at the inlet and outlet"; R20): rho and u
+ *                as above, Pi^neq = -rho tau c_s^2 (grad u + grad u^T) of the
+ *                new velocity field by second-order differences (one-sided
+ *                along the normal and at the face's edges, central elsewhere).
+ *                One rank, MOMENTS only (else MRLBM_ERR_UNSUPPORTED); >= 3
+ *                nodes along every non-periodic axis (else INVALID_ARGUMENT).
+ *                Runs as a separate face kernel after the fused step.
+ * Open faces (VELOCITY/PRESSURE[_FD]) are supported on the x and y faces of 3D
  * domains and on the x faces of 2D domains (not on the marching / slab axis). */
 typedef enum {
     MRLBM_PERIODIC = 0, MRLBM_WALL = 1, MRLBM_MOVING_WALL = 2,
-    MRLBM_VELOCITY = 3, MRLBM_PRESSURE = 4
+    MRLBM_VELOCITY = 3, MRLBM_PRESSURE = 4,
+    MRLBM_VELOCITY_FD = 5, MRLBM_PRESSURE_FD = 6
 } mrlbm_bc_kind;
 
 typedef struct {
     mrlbm_bc_kind kind;
     double u[3];             /* MOVING_WALL / VELOCITY (uniform) velocity */
     double rho;              /* PRESSURE density */
-    const double *u_profile; /* optional, VELOCITY only: [face nodes][D], host,
+    const double *u_profile; /* optional, VELOCITY[_FD] only: [face nodes][D], host,
                                 row-major over the two other axes (slower axis
                                 first; global, not slab-local); copied at create */
 } mrlbm_face;

@@ -59,6 +59,7 @@ struct Variant {
     void (*get)(const void *, double *, mr::GridArgs, cudaStream_t);
     void (*pops)(const void *, double *, mr::GridArgs, double, cudaStream_t);
     void (*finite)(const void *, mr::GridArgs, int *, cudaStream_t);
+    void (*fd)(const mr::FdArgs &, long long, cudaStream_t);
     const void *kernel_fn;
 };
 
@@ -93,6 +94,9 @@ template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB> Var
     v.finite = [](const void *buf, mr::GridArgs g, int *flag, cudaStream_t st) {
         mr::finite_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
             (const Real *)buf, g, flag);
+    };
+    v.fd = [](const mr::FdArgs &a, long long nodes, cudaStream_t st) {
+        mr::fd_face_kernel<LAT, Real><<<grid_for(nodes), 256, 0, st>>>(a);
     };
     return v;
 }
@@ -238,6 +242,7 @@ struct mrlbm_ctx {
     bool own_stream = false;
     cudaEvent_t ev_ready = nullptr, ev_comm = nullptr, ev_t0 = nullptr, ev_t1 = nullptr;
     double *prof_dev[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+    bool fd_face[4] = {false, false, false, false}; // kernel faces A-, A+, B-, B+ with the FD scheme (R20)
     double *io = nullptr;  // fp64 staging for set/get/populations
     size_t io_bytes = 0;
     int *flag = nullptr;
@@ -302,6 +307,25 @@ mrlbm_status enqueue_one_step(mrlbm_ctx *h, cudaStream_t st)
         h->kernels++;
     } else if (h->nranks == 1) {
         launch_range(h, src, 0, h->nC, st);
+        // finite-difference open faces: stress of the face nodes from the new velocity field
+        for (int K = 0; K < 4; K++) {
+            if (!h->fd_face[K]) continue;
+            mr::FdArgs f;
+            f.buf = node0(h, 1 - src);
+            f.nA = h->nA;
+            f.nB = h->nB;
+            f.nC = h->nC;
+            f.pitch = h->pitch;
+            f.mstride = h->mstride;
+            f.pstride = h->pstride;
+            f.face = K;
+            f.per[0] = h->base.kind[0] == mr::BC_PERIODIC;
+            f.per[1] = h->D == 3 && h->base.kind[2] == mr::BC_PERIODIC;
+            f.per[2] = h->base.wrapC;
+            f.tau = h->tau;
+            h->var.fd(f, (long long)(K < 2 ? h->nB : h->nA) * h->nC, st);
+            h->kernels++;
+        }
     } else {
         // halo exchange of the boundary planes of the current state, overlapped
         // with the interior layers [1, nC-1) that do not read the ghost planes
@@ -343,7 +367,11 @@ mrlbm_status ensure_io(mrlbm_ctx *h, size_t bytes)
 }
 
 bool is_wall(int k) { return k == MRLBM_WALL || k == MRLBM_MOVING_WALL; }
-bool is_open(int k) { return k == MRLBM_VELOCITY || k == MRLBM_PRESSURE; }
+bool is_open(int k) { return k == MRLBM_VELOCITY || k == MRLBM_PRESSURE || k == MRLBM_VELOCITY_FD || k == MRLBM_PRESSURE_FD; }
+bool is_fd(int k) { return k == MRLBM_VELOCITY_FD || k == MRLBM_PRESSURE_FD; }
+bool is_velocity(int k) { return k == MRLBM_VELOCITY || k == MRLBM_VELOCITY_FD; }
+// the fused kernel's face kind: FD faces take the regularized face's rho / u rule
+int kernel_kind(int k) { return k == MRLBM_VELOCITY_FD ? MRLBM_VELOCITY : (k == MRLBM_PRESSURE_FD ? MRLBM_PRESSURE : k); }
 
 } // namespace
 
@@ -430,7 +458,7 @@ mrlbm_status mrlbm_validate_repr(mrlbm_lattice lattice, int64_t nx, int64_t ny, 
     if (!bnd) return MRLBM_OK;
     for (int F = 0; F < 2 * D; F++) {
         const int k = bnd->face[F].kind;
-        if (k < MRLBM_PERIODIC || k > MRLBM_PRESSURE) return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown face kind");
+        if (k < MRLBM_PERIODIC || k > MRLBM_PRESSURE_FD) return fail(MRLBM_ERR_INVALID_ARGUMENT, "unknown face kind");
     }
     for (int ax = 0; ax < D; ax++) {
         const bool p0 = bnd->face[2 * ax].kind == MRLBM_PERIODIC, p1 = bnd->face[2 * ax + 1].kind == MRLBM_PERIODIC;
@@ -442,7 +470,19 @@ mrlbm_status mrlbm_validate_repr(mrlbm_lattice lattice, int64_t nx, int64_t ny, 
             return fail(MRLBM_ERR_INVALID_ARGUMENT, "moving-wall velocity must be tangential");
         if (f.kind == MRLBM_MOVING_WALL && D == 2 && f.u[2] != 0.0)
             return fail(MRLBM_ERR_INVALID_ARGUMENT, "2D moving-wall velocity has a z component");
-        if (f.kind == MRLBM_PRESSURE && !(f.rho > 0)) return fail(MRLBM_ERR_INVALID_ARGUMENT, "pressure face needs rho > 0");
+        if ((f.kind == MRLBM_PRESSURE || f.kind == MRLBM_PRESSURE_FD) && !(f.rho > 0))
+            return fail(MRLBM_ERR_INVALID_ARGUMENT, "pressure face needs rho > 0");
+    }
+    bool any_fd = false;
+    for (int F = 0; F < 2 * D; F++) any_fd |= is_fd(bnd->face[F].kind);
+    if (any_fd) {
+        if (repr != MRLBM_MOMENTS) return fail(MRLBM_ERR_UNSUPPORTED, "finite-difference faces need the moment representation");
+        if (nranks > 1) return fail(MRLBM_ERR_UNSUPPORTED, "finite-difference faces run on one rank");
+        // second-order one-sided stencils need 3 nodes along the normal and along non-periodic tangents
+        const int64_t ext[3] = {nx, ny, D == 3 ? nz : 1};
+        for (int ax = 0; ax < D; ax++)
+            if (bnd->face[2 * ax].kind != MRLBM_PERIODIC && ext[ax] < 3)
+                return fail(MRLBM_ERR_INVALID_ARGUMENT, "finite-difference faces need >= 3 nodes along bounded axes");
     }
     if (repr == MRLBM_DISTRIBUTIONS)
         for (int F = 0; F < 2 * D; F++)
@@ -596,7 +636,7 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     // velocity profiles -> device
     for (int F = 0; F < 2 * h->D; F++) {
         mrlbm_face &f = h->bnd.face[F];
-        if (f.kind == MRLBM_VELOCITY && f.u_profile) {
+        if (is_velocity(f.kind) && f.u_profile) {
             const int ax = F / 2;
             const size_t nodes = (size_t)(nx * ny * h->gn[2]) / (size_t)h->gn[ax];
             const size_t bytes = nodes * h->D * sizeof(double);
@@ -649,7 +689,8 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
             continue;
         }
         const mrlbm_face &f = h->bnd.face[phys[K]];
-        a.kind[K] = f.kind;
+        a.kind[K] = kernel_kind(f.kind);
+        if (K < 4) h->fd_face[K] = is_fd(f.kind);
         for (int q = 0; q < 3; q++) a.uw[K][q] = f.kind == MRLBM_MOVING_WALL ? f.u[q] : 0.0;
         if (K < 4) {
             a.open_drho[K] = f.rho - 1.0;

@@ -859,6 +859,88 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     }
 }
 
+// ------------------------------------------------------------ finite-difference open faces
+// Latt et al. [6] "FD" inlet / outlet (the paper's proxy apps; R20),
+// run after the fused step on the new state: the fused kernel has set rho and
+// u of the face nodes by the regularized rule (R14); this pass replaces their
+// stress by the Chapman-Enskog value of the new velocity field,
+//   Pi = rho u u - rho tau c_s^2 (d_a u_b + d_b u_a),
+// second-order differences: one-sided along the face normal and at the face's
+// edges, central elsewhere (wrapped on periodic axes).  Reads u, writes Pi of
+// face nodes only (plus their periodic ghost copies), so there is no hazard.
+struct FdArgs {
+    void *buf;          // node (0,0) of plane 0 of the state to update
+    int nA, nB, nC, pitch;
+    long long mstride, pstride;
+    int face;           // kernel face 0 A-, 1 A+, 2 B-, 3 B+
+    int per[3];         // periodic kernel axes A, B, C
+    double tau;
+};
+
+template <int LAT, typename Real> __global__ void fd_face_kernel(FdArgs g)
+{
+    using L = Lattice<LAT>;
+    constexpr int D = L::D;
+    Real *buf = reinterpret_cast<Real *>(g.buf);
+    const int ax = g.face / 2;                    // kernel axis of the face normal
+    const int n[3] = {g.nA, g.nB, g.nC};
+    const long long nodes = (long long)(ax == 0 ? g.nB : g.nA) * g.nC;
+    // kernel axis -> physical axis (2D: A = x, C = y; 3D: A = x, B = y, C = z)
+    const int phys[3] = {0, 1, D == 3 ? 2 : 1};
+    for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < nodes; t += (long long)gridDim.x * blockDim.x) {
+        int idx[3];
+        idx[2] = (int)(t / (ax == 0 ? g.nB : g.nA));
+        const int r = (int)(t % (ax == 0 ? g.nB : g.nA));
+        idx[ax] = (g.face % 2 == 0) ? 0 : n[ax] - 1;
+        idx[1 - ax] = r;
+        auto at = [&](int a, int b, int c) -> const Real * {
+            return buf + (long long)(c + 1) * g.pstride + (long long)b * g.pitch + a;
+        };
+        auto u_at = [&](const int (&q)[3], int comp) -> Real { return at(q[0], q[1], q[2])[(1 + comp) * g.mstride]; };
+        Real grad[3][3] = {}; // grad[a][b] = d_a u_b, physical axes
+#pragma unroll
+        for (int X = 0; X < 3; X++) {
+            if (D == 2 && X == 1) continue;
+            const int i = idx[X], nx = n[X];
+            int q0[3] = {idx[0], idx[1], idx[2]}, q1[3] = {idx[0], idx[1], idx[2]}, q2[3] = {idx[0], idx[1], idx[2]};
+            const bool central = g.per[X] || (i > 0 && i < nx - 1);
+            if (central) {
+                q1[X] = (i + 1) % nx;
+                q2[X] = (i - 1 + nx) % nx;
+            } else {
+                const int s = (i == 0) ? 1 : -1;
+                q1[X] = i + s;
+                q2[X] = i + 2 * s;
+            }
+#pragma unroll
+            for (int b = 0; b < D; b++) {
+                Real d;
+                if (central) d = Real(0.5) * (u_at(q1, b) - u_at(q2, b));
+                else d = Real(i == 0 ? 0.5 : -0.5) * (Real(-3) * u_at(q0, b) + Real(4) * u_at(q1, b) - u_at(q2, b));
+                grad[phys[X]][b] = d;
+            }
+        }
+        Real *node = buf + (long long)(idx[2] + 1) * g.pstride + (long long)idx[1] * g.pitch + idx[0];
+        const Real rho = Real(1) + node[0];
+        Real u[3] = {Real(0), Real(0), Real(0)};
+#pragma unroll
+        for (int b = 0; b < D; b++) u[b] = node[(1 + b) * g.mstride];
+        const Real k = -rho * Real(g.tau) * Real(1.0 / 3.0);
+        // periodic ghost copy of this face node (in-plane axis along the face)
+        long long goff = 0;
+        if (ax == 0 && D == 3 && g.per[1]) goff = idx[1] == 0 ? (long long)g.nB * g.pitch : (idx[1] == g.nB - 1 ? -(long long)g.nB * g.pitch : 0);
+        if (ax == 1 && g.per[0]) goff = idx[0] == 0 ? g.nA : (idx[0] == g.nA - 1 ? -g.nA : 0);
+#pragma unroll
+        for (int a = 0; a < D; a++)
+#pragma unroll
+            for (int b = a; b < D; b++) {
+                const Real v = fma(k, grad[a][b] + grad[b][a], rho * u[a] * u[b]);
+                node[pslot<D>(a, b) * g.mstride] = v;
+                if (goff) node[pslot<D>(a, b) * g.mstride + goff] = v;
+            }
+    }
+}
+
 // ------------------------------------------------------------ side kernels
 struct GridArgs {
     int nA, nB, nC, pitch;

@@ -27,7 +27,8 @@ LATTICES = {"D2Q9": 0, "D3Q19": 1, "D3Q27": 2}
 REGS = {"projective": 0, "recursive": 1, "bgk": 2}
 REPRS = {"moments": 0, "distributions": 1}
 PRECISIONS = {"fp64": 0, "fp32": 1}
-BC = {"periodic": 0, "wall": 1, "moving_wall": 2, "velocity": 3, "pressure": 4}
+BC = {"periodic": 0, "wall": 1, "moving_wall": 2, "velocity": 3, "pressure": 4,
+      "velocity_fd": 5, "pressure_fd": 6}
 FACES = ("x-", "x+", "y-", "y+", "z-", "z+")
 Q_OF = {"D2Q9": 9, "D3Q19": 19, "D3Q27": 27}
 M_OF = {"D2Q9": 6, "D3Q19": 10, "D3Q27": 10}

@@ -101,6 +101,24 @@ def test_validation_codes_distribution_representation():
     assert mrlbm.validate("D3Q19", 8, 8, 8, 0.5, "bgk", representation="distributions") == INV
 
 
+def test_validation_codes_fd_faces():
+    """Finite-difference faces (R20): one rank, moments only, >= 3 nodes along bounded axes."""
+    INV, UNS = -1, -2
+    b = walls(2)
+    b["x-"] = {"kind": "velocity_fd", "u": [0.01, 0, 0]}
+    b["x+"] = {"kind": "pressure_fd", "rho": 1.0}
+    assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, boundary=b) == 0
+    assert mrlbm.validate("D2Q9", 2, 8, 1, 0.6, boundary=b) == INV          # 2 nodes along the normal
+    assert mrlbm.validate("D2Q9", 8, 2, 1, 0.6, boundary=b) == INV          # 2 nodes along a walled tangent
+    assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, boundary=b, nranks=2) == UNS
+    assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, boundary=b, representation="distributions") == UNS
+    b["x+"] = {"kind": "pressure_fd", "rho": 0.0}
+    assert mrlbm.validate("D2Q9", 8, 8, 1, 0.6, boundary=b) == INV
+    b = {"y-": {"kind": "velocity_fd", "u": [0, 0.01, 0]}, "y+": {"kind": "pressure", "rho": 1.0}}
+    assert mrlbm.validate("D3Q19", 8, 8, 2, 0.6, boundary=b) == 0           # periodic x and z: no minimum
+    assert mrlbm.validate("D3Q19", 8, 8, 8, 0.6, boundary={"z-": {"kind": "velocity_fd"}, "z+": {"kind": "wall"}}) == UNS
+
+
 def test_create_fails_loudly_without_gpu():
     import torch
     if torch.cuda.is_available():
