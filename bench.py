@@ -243,7 +243,8 @@ def run_gpu(args, rank, world, local_rank):
     elif args.collision:
         c.regularization = args.collision
     nccl_id = None
-    if world > 1:
+    p2p = world > 1 and args.transport == "p2p"
+    if world > 1 and not p2p:
         idt = torch.zeros(128, dtype=torch.uint8, device=dev)
         if rank == 0:
             idt.copy_(torch.frombuffer(bytearray(mrlbm.nccl_unique_id()), dtype=torch.uint8).to(dev))
@@ -252,7 +253,13 @@ def run_gpu(args, rank, world, local_rank):
     stream = torch.cuda.Stream(device=dev)
     s = mrlbm.Solver(c.lattice, c.nx, c.ny, c.nz, c.tau, c.regularization, c.boundary, precision=c.precision,
                      device=local_rank, stream=stream.cuda_stream, rank=rank, nranks=world, nccl_id=nccl_id,
-                     representation="distributions" if st else "moments")
+                     representation="distributions" if st else "moments", transport="p2p" if p2p else "nccl")
+    if p2p:
+        # halo pushes through peer memory (CUDA IPC over NVLink): exchange the handles once
+        from paper_conf_sc_valero_laravgr23_b200 import distributed as sd
+        handles = [None] * world
+        dist.all_gather_object(handles, s.p2p_handle())
+        sd.p2p_connect(s, handles, sd.slab_axis_periodic(c.boundary, c.D))
     # initial state: this rank's slab of the seeded initial moments
     m0 = c.initial_moments()
     sl = slice(s.offset, s.offset + s.n_local)
@@ -333,7 +340,8 @@ def run_gpu(args, rank, world, local_rank):
     line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "f64" if c.precision == "fp64" else "f32", "data": "synthetic",
-            "config": dict(workload_config(c, world), method=args.method),
+            "config": dict(workload_config(c, world), method=args.method,
+                           **({"transport": args.transport} if world > 1 else {})),
             "per_gpu_mlups": value / world,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": tr, "peak_source": peak_src,
@@ -365,6 +373,8 @@ def main():
                     help="MR = the paper's moment representation (default); ST = its distribution baseline")
     ap.add_argument("--collision", default=None, choices=["projective", "recursive", "bgk"],
                     help="override the collision (ST default: bgk, the paper's Alg. 1)")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
+                    help="N > 1 halo transport: NCCL send/recv (default) or peer-memory pushes fused into the step")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--ref-side", type=int, default=1024, help="reference arm: max sample sub-domain side")

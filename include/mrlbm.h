@@ -67,6 +67,17 @@ typedef enum { MRLBM_MOMENTS = 0, MRLBM_DISTRIBUTIONS = 1 } mrlbm_representation
  * (P:L257); FP32 stores rho - 1 and shifted populations (R16). */
 typedef enum { MRLBM_FP64 = 0, MRLBM_FP32 = 1 } mrlbm_precision;
 
+/* Halo transport between z-slab ranks (nranks > 1):
+ *   NCCL  per step, ncclSend/ncclRecv of one boundary plane per face on a
+ *         communication stream, overlapped with the interior layers.
+ *   P2P   the fused step itself stores its first / last layer straight into
+ *         the neighbours' ghost planes through peer memory (CUDA IPC; NVLink
+ *         between GPUs), and device-side counters in peer memory order the
+ *         steps (no NCCL call, no separate copy).  Ranks may share a device
+ *         (then the peer "link" is local memory).  Requires
+ *         mrlbm_p2p_handle / mrlbm_p2p_connect before the first step. */
+typedef enum { MRLBM_TRANSPORT_NCCL = 0, MRLBM_TRANSPORT_P2P = 1 } mrlbm_transport;
+
 /* Face treatment ("bounceback ... at the channel walls", inlet/outlet
  * per Latt et al. [6]; readings R12-R14):
  *   PERIODIC     both faces of an axis must be periodic
@@ -114,6 +125,7 @@ typedef struct {
     const void *nccl_unique_id;/* 128-byte ncclUniqueId for nranks > 1 (one GPU per
                                   rank); NULL with nranks > 1 = slab-group mode */
     mrlbm_representation representation; /* default MOMENTS */
+    mrlbm_transport transport;  /* nranks > 1: halo transport, default NCCL (see below) */
 } mrlbm_options;
 
 typedef int mrlbm_status;
@@ -191,6 +203,22 @@ const char *mrlbm_last_error(void); /* thread-local detail of the last error */
 /* Write a 128-byte ncclUniqueId into id (rank 0 creates it, then it is
  * broadcast out of band, e.g. through torch.distributed). */
 mrlbm_status mrlbm_nccl_unique_id(void *id128);
+
+/* P2P transport setup (options.transport = MRLBM_TRANSPORT_P2P, nranks > 1).
+ * mrlbm_p2p_handle writes this rank's MRLBM_P2P_HANDLE_BYTES-byte handle
+ * (CUDA IPC handles of its two state buffers and its sync counters, plus raw
+ * pointers used when the neighbour lives in the same process) into blob;
+ * distribute them out of band (e.g. torch.distributed all_gather).
+ * mrlbm_p2p_connect maps the handles of the lower / upper z neighbour (NULL
+ * where the slab has none: non-periodic ends); both may be the same rank.
+ * Collective: every rank connects before any rank steps.  Errors:
+ * MRLBM_ERR_INVALID_ARGUMENT (not a P2P handle, wrong neighbour rank or
+ * layout), MRLBM_ERR_CUDA (IPC mapping failed).  A neighbour that stops
+ * stepping makes this rank's next step give up after 30 s; mrlbm_sync then
+ * returns MRLBM_ERR_CUDA. */
+#define MRLBM_P2P_HANDLE_BYTES 512
+mrlbm_status mrlbm_p2p_handle(mrlbm_t h, void *blob);
+mrlbm_status mrlbm_p2p_connect(mrlbm_t h, const void *blob_lo, const void *blob_hi);
 
 /* Slab-group mode (one process, one device): handles created with nranks = P,
  * rank = r and nccl_unique_id = NULL form one z-slab decomposition whose halo

@@ -12,6 +12,7 @@
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <cmath>
@@ -248,6 +249,14 @@ struct mrlbm_ctx {
     int *flag = nullptr;
     ncclComm_t comm = nullptr;
     bool group_mode = false;    // nranks > 1 without NCCL: ghosts filled by mrlbm_step_group
+    // P2P transport: peer memory pushes + device counters (mrlbm_p2p_*)
+    bool p2p = false, p2p_connected = false;
+    unsigned long long *sync = nullptr;            // [0] own pushes, [1] from lo, [2] from hi
+    int *p2p_err = nullptr;
+    void *peer_plane_lo[2] = {nullptr, nullptr};   // lower neighbour's HIGH ghost plane (start), per buffer
+    void *peer_plane_hi[2] = {nullptr, nullptr};   // upper neighbour's LOW ghost plane (start), per buffer
+    unsigned long long *peer_sync_lo = nullptr, *peer_sync_hi = nullptr;
+    std::vector<void *> ipc_opened;                // IPC mappings to close
     int nb_lo = -1, nb_hi = -1; // neighbour ranks along C (-1 none)
     cudaGraphExec_t graph[2] = {nullptr, nullptr};
     int graph_steps = 0;
@@ -279,12 +288,17 @@ mr::GridArgs grid_args(const mrlbm_ctx *h)
 }
 
 // launch the fused kernel over owned layers [cb, ce) reading buf[src]
-void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st)
+void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st, bool push = false)
 {
     if (ce <= cb) return;
     StepArgs a = h->base;
     a.src = node0(h, src);
     a.dst = node0(h, 1 - src);
+    if (push) { // P2P: layers 0 / nC-1 of the new state also go to the neighbours' ghost planes
+        const size_t org = (size_t)h->origin * h->wbytes;
+        a.peer_lo = h->peer_plane_lo[1 - src] ? (char *)h->peer_plane_lo[1 - src] + org : nullptr;
+        a.peer_hi = h->peer_plane_hi[1 - src] ? (char *)h->peer_plane_hi[1 - src] + org : nullptr;
+    }
     a.c_begin = cb;
     a.c_end = ce;
     const int span = ce - cb;
@@ -305,6 +319,18 @@ mrlbm_status enqueue_one_step(mrlbm_ctx *h, cudaStream_t st)
         dim3 grid((unsigned)((h->st_grid.nx + h->sv.BX - 1) / h->sv.BX), (unsigned)h->st_grid.ny, (unsigned)h->st_grid.nz);
         h->sv.step(a, grid, st);
         h->kernels++;
+    } else if (h->p2p) {
+        // P2P: interior layers need no ghost plane; then wait until both
+        // neighbours have pushed as often as this rank (our ghosts are current,
+        // and they are done reading the ghost planes we push into), run the
+        // boundary layers with the push fused into their stores, and signal
+        if (!h->p2p_connected) return fail(MRLBM_ERR_INVALID_ARGUMENT, "P2P transport: mrlbm_p2p_connect first");
+        launch_range(h, src, 1, h->nC - 1, st);
+        mr::p2p_wait_kernel<<<1, 1, 0, st>>>(h->sync, h->nb_lo >= 0, h->nb_hi >= 0, h->p2p_err);
+        launch_range(h, src, 0, 1, st, true);
+        launch_range(h, src, h->nC - 1, h->nC, st, true);
+        mr::p2p_signal_kernel<<<1, 1, 0, st>>>(h->sync, h->peer_sync_lo, h->peer_sync_hi);
+        h->kernels += 2;
     } else if (h->nranks == 1) {
         launch_range(h, src, 0, h->nC, st);
         // finite-difference open faces: stress of the face nodes from the new velocity field
@@ -363,6 +389,28 @@ mrlbm_status ensure_io(mrlbm_ctx *h, size_t bytes)
         return fail(MRLBM_ERR_OUT_OF_MEMORY, "staging allocation failed");
     }
     h->io_bytes = bytes;
+    return MRLBM_OK;
+}
+
+// P2P: after the state was set from outside, push its boundary planes into the
+// neighbours' ghost planes of the current buffer (ordered like a step's push)
+mrlbm_status p2p_prologue(mrlbm_ctx *h)
+{
+    if (!h->p2p || !h->p2p_connected) return MRLBM_OK;
+    const int b = h->cur;
+    char *base = (char *)h->buf[b];
+    const size_t plane = (size_t)h->pstride * h->wbytes;
+    mr::p2p_wait_kernel<<<1, 1, 0, h->stream>>>(h->sync, h->nb_lo >= 0, h->nb_hi >= 0, h->p2p_err);
+    if (h->prec == MRLBM_FP32)
+        mr::p2p_push_planes_kernel<float><<<grid_for(h->pstride), 256, 0, h->stream>>>(
+            (const float *)(base + plane), (const float *)(base + plane * h->nC), (float *)h->peer_plane_lo[b],
+            (float *)h->peer_plane_hi[b], h->pstride);
+    else
+        mr::p2p_push_planes_kernel<double><<<grid_for(h->pstride), 256, 0, h->stream>>>(
+            (const double *)(base + plane), (const double *)(base + plane * h->nC), (double *)h->peer_plane_lo[b],
+            (double *)h->peer_plane_hi[b], h->pstride);
+    mr::p2p_signal_kernel<<<1, 1, 0, h->stream>>>(h->sync, h->peer_sync_lo, h->peer_sync_hi);
+    MR_CUDA(cudaGetLastError());
     return MRLBM_OK;
 }
 
@@ -751,8 +799,18 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
         h->nseg = (int)((h->nC + seg - 1) / seg);
     }
 
-    h->group_mode = h->nranks > 1 && !o.nccl_unique_id;
-    if (h->nranks > 1 && !h->group_mode) {
+    h->p2p = h->nranks > 1 && o.transport == MRLBM_TRANSPORT_P2P;
+    h->group_mode = h->nranks > 1 && !h->p2p && !o.nccl_unique_id;
+    if (h->p2p) {
+        // own sync counters (IPC-exportable cudaMalloc allocation) and error flag
+        if (cudaMalloc(&h->sync, 4 * sizeof(unsigned long long)) != cudaSuccess ||
+            cudaMalloc(&h->p2p_err, sizeof(int)) != cudaSuccess)
+            return cleanup_fail(fail(MRLBM_ERR_OUT_OF_MEMORY, "p2p sync"));
+        if (cudaMemset(h->sync, 0, 4 * sizeof(unsigned long long)) != cudaSuccess ||
+            cudaMemset(h->p2p_err, 0, sizeof(int)) != cudaSuccess)
+            return cleanup_fail(fail(MRLBM_ERR_CUDA, "p2p sync init"));
+    }
+    if (h->nranks > 1 && !h->group_mode && !h->p2p) {
         if (cudaStreamCreateWithFlags(&h->comm_stream, cudaStreamNonBlocking) != cudaSuccess)
             return cleanup_fail(fail(MRLBM_ERR_CUDA, "comm stream"));
         ncclUniqueId id;
@@ -772,6 +830,9 @@ void mrlbm_destroy(mrlbm_t h)
     if (!h) return;
     if (h->stream) cudaStreamSynchronize(h->stream);
     if (h->comm) ncclCommDestroy(h->comm);
+    for (void *p : h->ipc_opened) cudaIpcCloseMemHandle(p);
+    if (h->sync) cudaFree(h->sync);
+    if (h->p2p_err) cudaFree(h->p2p_err);
     for (int i = 0; i < 2; i++)
         if (h->graph[i]) cudaGraphExecDestroy(h->graph[i]);
     for (int i = 0; i < 2; i++)
@@ -799,7 +860,7 @@ mrlbm_status mrlbm_set_moments_device(mrlbm_t h, const double *src_dev, int64_t 
     if (h->repr == MRLBM_DISTRIBUTIONS) h->sv.set(src_dev, h->buf[h->cur], h->st_grid, h->stream);
     else h->var.set(src_dev, node0(h, h->cur), grid_args(h), h->stream);
     MR_CUDA(cudaGetLastError());
-    return MRLBM_OK;
+    return p2p_prologue(h);
 }
 
 mrlbm_status mrlbm_get_moments_device(mrlbm_t h, double *dst_dev, int64_t count)
@@ -887,6 +948,8 @@ mrlbm_status mrlbm_set_populations(mrlbm_t h, const double *src, int64_t count)
         }
         MR_CUDA(cudaGetLastError());
         h->var.set(mom, node0(h, h->cur), grid_args(h), h->stream);
+        mrlbm_status ps = p2p_prologue(h);
+        if (ps) return ps;
     }
     MR_CUDA(cudaGetLastError());
     MR_CUDA(cudaStreamSynchronize(h->stream));
@@ -936,8 +999,105 @@ mrlbm_status mrlbm_sync(mrlbm_t h)
     if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
     MR_CUDA(cudaStreamSynchronize(h->stream));
     if (h->comm_stream) MR_CUDA(cudaStreamSynchronize(h->comm_stream));
+    if (h->p2p_err) {
+        int e = 0;
+        MR_CUDA(cudaMemcpy(&e, h->p2p_err, sizeof(int), cudaMemcpyDeviceToHost));
+        if (e) return fail(MRLBM_ERR_CUDA, "P2P transport: a neighbour stopped (wait timed out)");
+    }
     return MRLBM_OK;
 }
+
+// ---------------------------------------------------------------- P2P transport setup
+namespace {
+struct P2PBlob {
+    uint32_t magic;
+    int32_t pid, rank, nranks, nC, prec;
+    int64_t pstride, origin;
+    uint64_t raw[3];                 // buf[0], buf[1], sync (same-process peers)
+    cudaIpcMemHandle_t ipc[3];
+};
+constexpr uint32_t kP2PMagic = 0x4d52503250u; // "MRP2P"
+static_assert(sizeof(P2PBlob) <= MRLBM_P2P_HANDLE_BYTES, "P2P handle blob too large");
+} // namespace
+
+mrlbm_status mrlbm_p2p_handle(mrlbm_t h, void *blob)
+{
+    if (!h || !blob) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
+    if (!h->p2p) return fail(MRLBM_ERR_INVALID_ARGUMENT, "not a P2P-transport handle");
+    P2PBlob b;
+    memset(&b, 0, sizeof(b));
+    b.magic = kP2PMagic;
+    b.pid = (int32_t)getpid();
+    b.rank = h->rank;
+    b.nranks = h->nranks;
+    b.nC = h->nC;
+    b.prec = h->prec;
+    b.pstride = h->pstride;
+    b.origin = h->origin;
+    void *ptrs[3] = {h->buf[0], h->buf[1], h->sync};
+    for (int i = 0; i < 3; i++) {
+        b.raw[i] = (uint64_t)(uintptr_t)ptrs[i];
+        MR_CUDA(cudaIpcGetMemHandle(&b.ipc[i], ptrs[i]));
+    }
+    memset(blob, 0, MRLBM_P2P_HANDLE_BYTES);
+    memcpy(blob, &b, sizeof(b));
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_p2p_connect(mrlbm_t h, const void *blob_lo, const void *blob_hi)
+{
+    if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
+    if (!h->p2p) return fail(MRLBM_ERR_INVALID_ARGUMENT, "not a P2P-transport handle");
+    if ((h->nb_lo >= 0) != (blob_lo != nullptr) || (h->nb_hi >= 0) != (blob_hi != nullptr))
+        return fail(MRLBM_ERR_INVALID_ARGUMENT, "neighbour handles do not match the slab's neighbours");
+    MR_CUDA(cudaSetDevice(h->device));
+    const size_t plane = (size_t)h->pstride * h->wbytes;
+    struct Mapped { int rank; void *p[3]; };
+    std::vector<Mapped> done;
+    auto map = [&](const void *blob, int want_rank, Mapped &out, int &nC) -> mrlbm_status {
+        P2PBlob b;
+        memcpy(&b, blob, sizeof(b));
+        if (b.magic != kP2PMagic || b.rank != want_rank || b.nranks != h->nranks || b.prec != h->prec ||
+            b.pstride != h->pstride || b.origin != h->origin)
+            return fail(MRLBM_ERR_INVALID_ARGUMENT, "P2P handle of the wrong rank or layout");
+        nC = b.nC;
+        for (const Mapped &m : done)
+            if (m.rank == want_rank) { out = m; return MRLBM_OK; }
+        out.rank = want_rank;
+        for (int i = 0; i < 3; i++) {
+            if (b.pid == (int32_t)getpid()) {
+                out.p[i] = (void *)(uintptr_t)b.raw[i];
+            } else {
+                void *p = nullptr;
+                cudaError_t e = cudaIpcOpenMemHandle(&p, b.ipc[i], cudaIpcMemLazyEnablePeerAccess);
+                if (e != cudaSuccess) return fail(MRLBM_ERR_CUDA, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+                h->ipc_opened.push_back(p);
+                out.p[i] = p;
+            }
+        }
+        done.push_back(out);
+        return MRLBM_OK;
+    };
+    if (blob_lo) {
+        Mapped m;
+        int nC = 0;
+        mrlbm_status s = map(blob_lo, h->nb_lo, m, nC);
+        if (s) return s;
+        for (int i = 0; i < 2; i++) h->peer_plane_lo[i] = (char *)m.p[i] + plane * (size_t)(nC + 1); // its high ghost
+        h->peer_sync_lo = (unsigned long long *)m.p[2];
+    }
+    if (blob_hi) {
+        Mapped m;
+        int nC = 0;
+        mrlbm_status s = map(blob_hi, h->nb_hi, m, nC);
+        if (s) return s;
+        for (int i = 0; i < 2; i++) h->peer_plane_hi[i] = m.p[i]; // its low ghost plane 0
+        h->peer_sync_hi = (unsigned long long *)m.p[2];
+    }
+    h->p2p_connected = true;
+    return MRLBM_OK;
+}
+
 
 mrlbm_status mrlbm_check_finite(mrlbm_t h)
 {

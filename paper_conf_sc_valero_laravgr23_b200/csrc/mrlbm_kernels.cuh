@@ -50,6 +50,11 @@ struct StepArgs {
     double open_u[4][3];    // VELOCITY faces: uniform velocity
     const double *open_prof[4]; // VELOCITY faces: optional [face nodes][D] (global)
     double omega;           // 1 - 1/tau
+    // P2P transport (peer memory over NVLink): node (0,0) of the lower / upper
+    // neighbour's ghost plane in its copy of this step's destination buffer.
+    // Layer 0 / nC-1 of the new state is pushed there as it is finalized, so
+    // the halo exchange rides on the stores of the fused step (null: no push)
+    void *peer_lo, *peer_hi;
 };
 
 // ------------------------------------------------------------ PTX helpers
@@ -723,18 +728,28 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         }
         if (!owner) return;
         Real *o = dst_node + (long long)(c + 1) * p.pstride;
+        auto store_plane = [&](Real *o) {
 #pragma unroll
-        for (int q = 0; q < M; q++) o[q * p.mstride] = out[q];
-        // periodic ghost copies of edge nodes (also the corner ghosts)
-        if (gA | gB) {
-            auto put = [&](int da, int db) {
-                Real *g = o + (long long)db * p.pitch + da;
+            for (int q = 0; q < M; q++) o[q * p.mstride] = out[q];
+            // periodic ghost copies of edge nodes (also the corner ghosts)
+            if (gA | gB) {
+                auto put = [&](int da, int db) {
+                    Real *g = o + (long long)db * p.pitch + da;
 #pragma unroll
-                for (int q = 0; q < M; q++) g[q * p.mstride] = out[q];
-            };
-            if (gA) put(gA, 0);
-            if (gB) put(0, gB);
-            if (gA && gB) put(gA, gB);
+                    for (int q = 0; q < M; q++) g[q * p.mstride] = out[q];
+                };
+                if (gA) put(gA, 0);
+                if (gB) put(0, gB);
+                if (gA && gB) put(gA, gB);
+            }
+        };
+        store_plane(o);
+        // P2P halo push: the slab's first / last layer also goes straight into
+        // the neighbour's ghost plane (peer memory), same in-plane layout
+        void *peer = (c == 0) ? p.peer_lo : ((c == nC - 1) ? p.peer_hi : nullptr);
+        if (peer) {
+            store_plane(reinterpret_cast<Real *>(peer) + (long long)b * p.pitch + a);
+            __threadfence_system();
         }
     };
 
@@ -939,6 +954,66 @@ template <int LAT, typename Real> __global__ void fd_face_kernel(FdArgs g)
                 if (goff) node[pslot<D>(a, b) * g.mstride + goff] = v;
             }
     }
+}
+
+// ------------------------------------------------------------ P2P transport synchronisation
+// Per handle, a device word array sync[4]: [0] pushes completed by this rank,
+// [1] / [2] pushes completed by the lower / upper neighbour (written by them,
+// through peer memory).  Before a step's boundary layers a rank waits until
+// both neighbours have completed as many pushes as itself: then its ghost
+// planes hold their latest layers (read after write) and they have finished
+// the step that last read the ghost planes it is about to overwrite (write
+// after read).  Device-side counters, so the sequence is graph-capturable.
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v)
+{
+    asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long globaltimer_ns()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
+__global__ void p2p_wait_kernel(unsigned long long *sync, int need_lo, int need_hi, int *err)
+{
+    const unsigned long long target = sync[0];
+    const unsigned long long t0 = globaltimer_ns();
+    while ((need_lo && ld_acquire_sys(&sync[1]) < target) || (need_hi && ld_acquire_sys(&sync[2]) < target)) {
+        __nanosleep(256);
+        if (globaltimer_ns() - t0 > 30ull * 1000000000ull) { // a neighbour stopped: report, do not hang
+            atomicExch(err, 2);
+            return;
+        }
+    }
+}
+
+__global__ void p2p_signal_kernel(unsigned long long *sync, unsigned long long *lo_sync, unsigned long long *hi_sync)
+{
+    __threadfence_system();
+    const unsigned long long c = sync[0] + 1;
+    sync[0] = c;
+    if (lo_sync) st_release_sys(&lo_sync[2], c); // this rank is its lower neighbour's upper neighbour
+    if (hi_sync) st_release_sys(&hi_sync[1], c);
+}
+
+// Prologue push after the state was set from outside: whole planes (pads and
+// in-plane ghosts included) into the neighbours' ghost planes.
+template <typename Real>
+__global__ void p2p_push_planes_kernel(const Real *own_first, const Real *own_last, Real *peer_lo, Real *peer_hi,
+                                       long long count)
+{
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < count; i += (long long)gridDim.x * blockDim.x) {
+        if (peer_lo) peer_lo[i] = own_first[i];
+        if (peer_hi) peer_hi[i] = own_last[i];
+    }
+    __threadfence_system();
 }
 
 // ------------------------------------------------------------ side kernels

@@ -35,3 +35,25 @@ def gather_slabs(local: np.ndarray, n_global: int, group=None) -> np.ndarray:
     out = [torch.empty_like(t) for _ in range(world)]
     dist.all_gather(out, t, group=group)
     return np.concatenate([o.numpy()[:, :shapes[r]] for r, o in enumerate(out)], axis=1)
+
+
+def slab_neighbours(nranks: int, rank: int, periodic: bool):
+    """(lower, upper) neighbour ranks along the slab axis, None at a bounded end
+    (the library's own rule: periodic slab axis wraps rank 0 <-> rank P-1)."""
+    lo = rank - 1 if rank > 0 else (nranks - 1 if periodic else None)
+    hi = rank + 1 if rank < nranks - 1 else (0 if periodic else None)
+    return lo, hi
+
+
+def slab_axis_periodic(boundary: dict | None, D: int) -> bool:
+    """Missing faces are periodic (include/mrlbm.h); the slab axis is z (3D) / y (2D)."""
+    face = "z-" if D == 3 else "y-"
+    spec = (boundary or {}).get(face)
+    return spec is None or spec.get("kind", "periodic") == "periodic"
+
+
+def p2p_connect(solver, handles: list, periodic: bool):
+    """Connect a P2P-transport solver to its slab neighbours, given every rank's
+    mrlbm_p2p_handle blob (e.g. from torch.distributed.all_gather_object)."""
+    lo, hi = slab_neighbours(len(handles), solver.rank, periodic)
+    solver.p2p_connect(handles[lo] if lo is not None else None, handles[hi] if hi is not None else None)

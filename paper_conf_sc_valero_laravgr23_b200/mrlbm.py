@@ -27,6 +27,8 @@ LATTICES = {"D2Q9": 0, "D3Q19": 1, "D3Q27": 2}
 REGS = {"projective": 0, "recursive": 1, "bgk": 2}
 REPRS = {"moments": 0, "distributions": 1}
 PRECISIONS = {"fp64": 0, "fp32": 1}
+TRANSPORTS = {"nccl": 0, "p2p": 1}
+P2P_HANDLE_BYTES = 512  # MRLBM_P2P_HANDLE_BYTES
 BC = {"periodic": 0, "wall": 1, "moving_wall": 2, "velocity": 3, "pressure": 4,
       "velocity_fd": 5, "pressure_fd": 6}
 FACES = ("x-", "x+", "y-", "y+", "z-", "z+")
@@ -37,7 +39,8 @@ M_OF = {"D2Q9": 6, "D3Q19": 10, "D3Q27": 10}
 API = ("mrlbm_default_options", "mrlbm_create", "mrlbm_set_moments", "mrlbm_step", "mrlbm_get_moments",
        "mrlbm_get_populations", "mrlbm_set_moments_device", "mrlbm_get_moments_device", "mrlbm_sync",
        "mrlbm_check_finite", "mrlbm_query", "mrlbm_launch_count", "mrlbm_time_steps", "mrlbm_destroy",
-       "mrlbm_status_string", "mrlbm_last_error", "mrlbm_nccl_unique_id", "mrlbm_set_populations")
+       "mrlbm_status_string", "mrlbm_last_error", "mrlbm_nccl_unique_id", "mrlbm_set_populations",
+       "mrlbm_p2p_handle", "mrlbm_p2p_connect")
 HOST_HELPERS = ("mrlbm_partition", "mrlbm_validate", "mrlbm_validate_repr", "mrlbm_kernel_config", "mrlbm_step_group")
 
 
@@ -53,7 +56,7 @@ class Boundary(ctypes.Structure):
 class Options(ctypes.Structure):
     _fields_ = [("precision", ctypes.c_int), ("device", ctypes.c_int), ("cuda_stream", ctypes.c_void_p),
                 ("rank", ctypes.c_int), ("nranks", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p),
-                ("representation", ctypes.c_int)]
+                ("representation", ctypes.c_int), ("transport", ctypes.c_int)]
 
 
 def _load():
@@ -89,6 +92,8 @@ def _load():
                                                ctypes.POINTER(Boundary), ctypes.c_int, ctypes.c_int]),
         "mrlbm_kernel_config": (ctypes.c_int, [vp, ip, ip, ip, ip, ip, ip, i64p]),
         "mrlbm_step_group": (ctypes.c_int, [ctypes.POINTER(vp), ctypes.c_int, i64]),
+        "mrlbm_p2p_handle": (ctypes.c_int, [vp, vp]),
+        "mrlbm_p2p_connect": (ctypes.c_int, [vp, vp, vp]),
     }
     for name, (res, args) in sig.items():
         fn = getattr(L, name)
@@ -170,9 +175,10 @@ class Solver:
 
     def __init__(self, lattice, nx, ny, nz=1, tau=0.6, regularization="projective", boundary=None,
                  precision="fp64", device=-1, stream=None, rank=0, nranks=1, nccl_id: bytes | None = None,
-                 representation="moments"):
+                 representation="moments", transport="nccl"):
         self.lattice, self.regularization, self.precision = lattice, regularization, precision
         self.representation = representation
+        self.rank, self.nranks = rank, nranks
         self.D = 2 if lattice == "D2Q9" else 3
         self.M, self.Q = M_OF[lattice], Q_OF[lattice]
         self.nx, self.ny, self.nz = nx, ny, (nz if self.D == 3 else 1)
@@ -185,6 +191,7 @@ class Solver:
         o.cuda_stream = stream
         o.rank, o.nranks = rank, nranks
         o.representation = REPRS[representation]
+        o.transport = TRANSPORTS[transport]
         if nccl_id is not None:
             self._id = ctypes.create_string_buffer(bytes(nccl_id), 128)
             o.nccl_unique_id = ctypes.cast(self._id, ctypes.c_void_p)
@@ -252,6 +259,21 @@ class Solver:
 
     def step(self, n=1):
         _check(lib.mrlbm_step(self._h, int(n)), "mrlbm_step")
+
+    # ---- P2P transport (transport="p2p", nranks > 1)
+    def p2p_handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(P2P_HANDLE_BYTES)
+        _check(lib.mrlbm_p2p_handle(self._h, ctypes.cast(buf, ctypes.c_void_p)), "mrlbm_p2p_handle")
+        return buf.raw
+
+    def p2p_connect(self, lo: bytes | None, hi: bytes | None):
+        """map the lower / upper neighbour's handle (None where the slab has none)"""
+        bl = ctypes.create_string_buffer(bytes(lo), P2P_HANDLE_BYTES) if lo is not None else None
+        bh = ctypes.create_string_buffer(bytes(hi), P2P_HANDLE_BYTES) if hi is not None else None
+        self._p2p_keep = (bl, bh)
+        _check(lib.mrlbm_p2p_connect(self._h, ctypes.cast(bl, ctypes.c_void_p) if bl is not None else None,
+                                     ctypes.cast(bh, ctypes.c_void_p) if bh is not None else None),
+               "mrlbm_p2p_connect")
 
     def sync(self):
         _check(lib.mrlbm_sync(self._h), "mrlbm_sync")

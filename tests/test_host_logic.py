@@ -146,3 +146,14 @@ def test_bench_workloads():
         assert (c5.lattice, c5.regularization, c5.nx, c5.ny, c5.nz) == ("D3Q19", "recursive", 1024, 1024, 128 * world)
         assert c5.boundary["x-"]["u_profile"].shape == (128 * world, 1024, 3)
     assert "channel" in bench.workload_config(bench.build_config("C5", "fp64", 1), 1)["workload"]
+
+
+def test_slab_neighbours_and_p2p_guards():
+    from paper_conf_sc_valero_laravgr23_b200 import distributed
+    assert distributed.slab_neighbours(4, 0, False) == (None, 1)
+    assert distributed.slab_neighbours(4, 3, False) == (2, None)
+    assert distributed.slab_neighbours(4, 0, True) == (3, 1)
+    assert distributed.slab_neighbours(2, 1, True) == (0, 0)
+    assert distributed.slab_axis_periodic({}, 3) and distributed.slab_axis_periodic({"x-": {"kind": "wall"}}, 2)
+    assert not distributed.slab_axis_periodic({"z-": {"kind": "wall"}}, 3)
+    assert mrlbm.TRANSPORTS == {"nccl": 0, "p2p": 1} and mrlbm.P2P_HANDLE_BYTES == 512
