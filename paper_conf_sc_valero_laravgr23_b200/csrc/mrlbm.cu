@@ -56,6 +56,8 @@ struct Variant {
     int TA, TB, S, BW;
     size_t smem;
     void (*step)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t);
+    void (*step_push)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t); // P2P boundary layers (or null)
+    const void *kernel_fn_push;
     void (*set)(const double *, void *, mr::GridArgs, cudaStream_t);
     void (*get)(const void *, double *, mr::GridArgs, cudaStream_t);
     void (*pops)(const void *, double *, mr::GridArgs, double, cudaStream_t);
@@ -66,7 +68,7 @@ struct Variant {
 
 inline int grid_for(long long n) { return (int)std::min<long long>((n + 255) / 256, 148LL * 16); }
 
-template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB> Variant make_variant()
+template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB, bool WITH_PUSH = false> Variant make_variant()
 {
     using L = mr::Lattice<LAT>;
     using SM = mr::StepSmem<LAT, Real, TA, TB, S>;
@@ -80,6 +82,14 @@ template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB> Var
     v.step = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
         mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB><<<grid, TA * TB, SM::bytes, st>>>(map, a);
     };
+    v.step_push = nullptr;
+    v.kernel_fn_push = nullptr;
+    if constexpr (WITH_PUSH) {
+        v.kernel_fn_push = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true>;
+        v.step_push = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
+            mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true><<<grid, TA * TB, SM::bytes, st>>>(map, a);
+        };
+    }
     v.set = [](const double *in, void *buf, mr::GridArgs g, cudaStream_t st) {
         mr::set_moments_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
             in, (Real *)buf, g);
@@ -113,7 +123,7 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile)
         if (tile == 1) return make_variant<LAT, REC, Real, 128, 1, 4, 4>();
         if (tile == 2) return make_variant<LAT, REC, Real, 128, 1, 6, 4>();
         if (tile == 3) return make_variant<LAT, REC, Real, 128, 1, 8, 3>();
-        return make_variant<LAT, REC, Real, 128, 1, 4, 5>();
+        return make_variant<LAT, REC, Real, 128, 1, 4, 5, true>();
     } else {
         constexpr bool f64 = sizeof(Real) == 8;
         // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
@@ -122,8 +132,10 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile)
         // TMA ring depth: with the A-movers exchanged by shuffles the fp64 32x8
         // tile fits three stages at two CTAs per SM; the 32x16 tile (one CTA
         // per SM) takes four in fp32
-        if (tile == 1 || small_only) return make_variant<LAT, REC, Real, 32, 8, 3, 2>();
-        return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 4), 1>();
+        // the library defaults also carry the P2P push instance
+        constexpr bool small_default = LAT == mr::LAT_D3Q19 || small_only;
+        if (tile == 1 || small_only) return make_variant<LAT, REC, Real, 32, 8, 3, 2, small_default>();
+        return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 4), 1, !small_default>();
     }
 }
 
@@ -305,7 +317,8 @@ void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st, bool p
     a.seg_len = std::min(h->seg_len, span);
     const int nseg = (span + a.seg_len - 1) / a.seg_len;
     dim3 grid(h->tilesA * h->tilesB, nseg);
-    h->var.step(h->tmap[src], a, grid, st);
+    if (push) h->var.step_push(h->tmap[src], a, grid, st);
+    else h->var.step(h->tmap[src], a, grid, st);
     h->kernels++;
 }
 
@@ -696,11 +709,15 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     }
 
     h->var = select_variant(lattice, reg, o.precision, env_int("MRLBM_TILE", 0));
-    if (cudaFuncSetAttribute(h->var.kernel_fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)h->var.smem) !=
-            cudaSuccess ||
-        cudaFuncSetAttribute(h->var.kernel_fn, cudaFuncAttributePreferredSharedMemoryCarveout,
-                             (int)cudaSharedmemCarveoutMaxShared) != cudaSuccess)
-        return cleanup_fail(fail(MRLBM_ERR_CUDA, "smem attribute"));
+    for (const void *fn : {h->var.kernel_fn, h->var.kernel_fn_push}) {
+        if (!fn) continue;
+        if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)h->var.smem) != cudaSuccess ||
+            cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                 (int)cudaSharedmemCarveoutMaxShared) != cudaSuccess)
+            return cleanup_fail(fail(MRLBM_ERR_CUDA, "smem attribute"));
+    }
+    if (o.transport == MRLBM_TRANSPORT_P2P && o.nranks > 1 && !h->var.step_push)
+        return cleanup_fail(fail(MRLBM_ERR_UNSUPPORTED, "P2P transport needs the default tile (MRLBM_TILE unset)"));
 
     // TMA descriptors: tensor {nA, nB, M, nC + 2} of the [plane][m][b][a] layout
     for (int i = 0; i < 2; i++) {

@@ -572,6 +572,15 @@ __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> finalize_open(RVec<Real, 
 // roles, except D3Q27 recursive, whose body unrolled twice spills registers
 template <int LAT, bool REC> struct Sweep {
     static constexpr bool two_set = !(LAT == LAT_D3Q27 && REC);
+    // a second, boundary-free body for interior CTAs (2D; the 3D bodies are
+    // large enough that two of them compete for the instruction cache)
+#if defined(MRLBM_NO_FAST_PATH)
+    static constexpr bool fast_path = false;
+#elif defined(MRLBM_FAST_PATH_3D)
+    static constexpr bool fast_path = true;
+#else
+    static constexpr bool fast_path = LAT == LAT_D2Q9;
+#endif
 };
 
 // exchange-plane slot of population k, or -1 if it does not go through shared
@@ -600,7 +609,9 @@ template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
     static constexpr size_t bytes = (S * stage_elems + 2 * F_elems) * sizeof(Real) + S * sizeof(uint64_t) + 128;
 };
 
-template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB>
+// PUSH: the P2P-transport instance for a rank's boundary layers (peer stores);
+// the plain instance carries none of that code
+template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB, bool PUSH = false>
 __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_constant__ CUtensorMap tmap,
                                                             const StepArgs p)
 {
@@ -634,35 +645,44 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     const int clast = (c1 < nC || p.hi_nb) ? c1 : c1 - 1;
     const int nl = clast - cfirst + 1;
 
+    // Fast CTAs: the whole window lies inside the domain, no owner sits on a
+    // domain face or a periodic edge, and the segment holds neither the first
+    // nor the last layer -- no wall, open face, ghost copy or peer push can
+    // occur, so that body is compiled without any of their tests (most CTAs)
+    const bool fast_cta = Sweep<LAT, REC>::fast_path && a0 >= 0 && a0 + TA <= nA &&
+                          (D == 2 || (b0 >= 0 && b0 + TB <= nB)) && c0 > 0 && c1 < nC;
+    auto run = [&](auto fast_tag) {
+    constexpr bool FAST = decltype(fast_tag)::value;
+
     // ---- per-thread roles
     const bool perA = p.kind[0] == BC_PERIODIC, perB = p.kind[2] == BC_PERIODIC;
     const bool inA = a >= 0 && a < nA, inB = b >= 0 && b < nB;
     // a window position holds a real node if it is inside the domain or is the
     // periodic ghost column / row (a = -1, nA; b = -1, nB), whose storage the
     // owning edge nodes refresh at every store (see store_ghosts)
-    const bool valid = (inA || (perA && (a == -1 || a == nA))) && (inB || (perB && (b == -1 || b == nB)));
+    const bool valid = FAST || ((inA || (perA && (a == -1 || a == nA))) && (inB || (perB && (b == -1 || b == nB))));
     const bool interior = tx >= 1 && tx < TA - 1 && ty >= HB && ty < TB - HB;
-    const bool owner = interior && inA && inB;
+    const bool owner = FAST ? interior : (interior && inA && inB);
     // SHFL: every lane of an interior row runs the streaming code (a warp is one
     // row, so the shuffles see all 32 lanes); only owners store
     const bool stream_lane = SHFL ? (ty >= HB && ty < TB - HB) : owner;
     // open faces in this CTA's window (CTA-uniform, so that the weighted and the
     // plain streaming bodies never diverge inside a warp)
     const int tilesB_ = gridDim.x / p.tilesA;
-    const bool cta_open = (p.kind[0] >= BC_VELOCITY && tA == 0) || (p.kind[1] >= BC_VELOCITY && tA == p.tilesA - 1) ||
-                          (D == 3 && ((p.kind[2] >= BC_VELOCITY && tB == 0) ||
-                                      (p.kind[3] >= BC_VELOCITY && tB == tilesB_ - 1)));
+    const bool cta_open = !FAST && ((p.kind[0] >= BC_VELOCITY && tA == 0) || (p.kind[1] >= BC_VELOCITY && tA == p.tilesA - 1) ||
+                                    (D == 3 && ((p.kind[2] >= BC_VELOCITY && tB == 0) ||
+                                                (p.kind[3] >= BC_VELOCITY && tB == tilesB_ - 1))));
     // ghost shift of an owner on a periodic edge: a = 0 -> column nA, a = nA-1 -> column -1
-    const int gA = !perA ? 0 : (a == 0 ? nA : (a == nA - 1 ? -nA : 0));
+    const int gA = (FAST || !perA) ? 0 : (a == 0 ? nA : (a == nA - 1 ? -nA : 0));
     const int gB = (D == 2 || !perB) ? 0 : (b == 0 ? nB : (b == nB - 1 ? -nB : 0));
     // pull-source availability along A/B: source at a-1 (c_a = +1), a+1 (c_a = -1)
     // walls touching this node in-plane (-1 lower face, +1 upper face)
     auto is_wall = [](int k) { return k == BC_WALL || k == BC_MOVING; };
-    const int bbA = (a == 0 && is_wall(p.kind[0])) ? -1 : ((a == nA - 1 && is_wall(p.kind[1])) ? 1 : 0);
+    const int bbA = FAST ? 0 : ((a == 0 && is_wall(p.kind[0])) ? -1 : ((a == nA - 1 && is_wall(p.kind[1])) ? 1 : 0));
     const int bbB = (D == 2) ? 0 : ((b == 0 && is_wall(p.kind[2])) ? -1 : ((b == nB - 1 && is_wall(p.kind[3])) ? 1 : 0));
     // open face of this node (index 0..3 into open_*), inward normal (physical x / y)
     int openF = -1, nx_in = 0, ny_in = 0;
-    if (owner) {
+    if (!FAST && owner) {
         if (a == 0 && p.kind[0] >= BC_VELOCITY) { openF = 0; nx_in = 1; }
         else if (a == nA - 1 && p.kind[1] >= BC_VELOCITY) { openF = 1; nx_in = -1; }
         else if (D == 3 && b == 0 && p.kind[2] >= BC_VELOCITY) { openF = 2; ny_in = 1; }
@@ -746,10 +766,12 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         store_plane(o);
         // P2P halo push: the slab's first / last layer also goes straight into
         // the neighbour's ghost plane (peer memory), same in-plane layout
-        void *peer = (c == 0) ? p.peer_lo : ((c == nC - 1) ? p.peer_hi : nullptr);
-        if (peer) {
-            store_plane(reinterpret_cast<Real *>(peer) + (long long)b * p.pitch + a);
-            __threadfence_system();
+        if constexpr (PUSH && !FAST) {
+            void *peer = (c == 0) ? p.peer_lo : ((c == nC - 1) ? p.peer_hi : nullptr);
+            if (peer) {
+                store_plane(reinterpret_cast<Real *>(peer) + (long long)b * p.pitch + a);
+                __threadfence_system();
+            }
         }
     };
 
@@ -798,7 +820,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         }
 
         if (stream_lane) {
-            const int bbC = (c == 0 && !p.lo_nb) ? -1 : ((c == nC - 1 && !p.hi_nb) ? 1 : 0);
+            const int bbC = FAST ? 0 : ((c == 0 && !p.lo_nb) ? -1 : ((c == nC - 1 && !p.hi_nb) ? 1 : 0));
             auto body = [&](auto open_tag) {
                 constexpr bool OPEN = decltype(open_tag)::value;
                 auto wt = [&](int kx, int ky) -> Real {
@@ -872,6 +894,9 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         }
         if (owner && clast == c1 - 1) finalize_store(accA, c1 - 1);
     }
+    };
+    if (fast_cta) run(std::true_type{});
+    else run(std::false_type{});
 }
 
 // ------------------------------------------------------------ finite-difference open faces
