@@ -143,3 +143,32 @@ def test_set_get_roundtrip(lat, precision):
         assert np.array_equal(got, m0)
     else:
         assert np.allclose(got, m0, rtol=1e-6, atol=1e-7)
+
+
+def fast_ctas(cfg, nA, nC):
+    """CTAs that take the boundary-free body (mrlbm_step_kernel: window
+    inside the domain along A, segment holding neither the first nor the
+    last layer along C) -- 2D only."""
+    TA, L = cfg["TA"], cfg["seg_len"]
+    tiles = [-1 + i * (TA - 2) for i in range(cfg["grid_x"])]
+    nA_fast = sum(1 for a0 in tiles if a0 >= 0 and a0 + TA <= nA)
+    segs = [(s * L, min(nC, (s + 1) * L) - 1) for s in range(cfg["grid_y"])]
+    return nA_fast * sum(1 for c0, c1 in segs if c0 > 0 and c1 < nC - 1)
+
+
+@pytest.mark.parametrize("precision", ["fp64", "fp32"])
+@pytest.mark.parametrize("reg", ["projective", "recursive"])
+@pytest.mark.parametrize("bc", ["periodic", "cavity"])
+def test_interior_fast_body(bc, reg, precision):
+    """A D2Q9 grid wide and tall enough that interior CTAs take the
+    boundary-free body (4 tiles along x, several segments along y), next to
+    boundary CTAs of every kind; element-by-element vs the oracle."""
+    from paper_conf_sc_valero_laravgr23_b200 import mrlbm
+    nx, ny = 400, 120
+    m0 = inputs.smooth_state(2, nx, ny, 1, U=0.05)
+    b = {} if bc == "periodic" else walls(2, ("y+", [0.1, 0.0, 0.0]))
+    with mrlbm.Solver("D2Q9", nx, ny, 1, 0.6, reg, b, precision=precision) as s:
+        cfg = s.kernel_config()
+    assert fast_ctas(cfg, nx, ny) > 0, cfg
+    errs, _, _ = run_pair("D2Q9", reg, nx, ny, 1, 0.6, b, m0, 500, precision)
+    assert_parity(errs, precision, f"D2Q9-{reg} {bc} interior body")
