@@ -10,8 +10,9 @@ PKG = Path(__file__).resolve().parent
 ROOT = PKG.parent
 CSRC = PKG / "csrc"
 LIB = PKG / "libmrlbm.so"
-SOURCES = [CSRC / "mrlbm.cu"]
-DEPS = SOURCES + [CSRC / "mrlbm_kernels.cuh", CSRC / "lattice.cuh", ROOT / "include" / "mrlbm.h"]
+# one translation unit per lattice (compiled in parallel) + the host / ABI unit
+SOURCES = [CSRC / "mrlbm.cu", CSRC / "var_d2q9.cu", CSRC / "var_d3q19.cu", CSRC / "var_d3q27.cu", CSRC / "var_st.cu"]
+DEPS = SOURCES + sorted(CSRC.glob("*.cuh")) + [ROOT / "include" / "mrlbm.h"]
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
@@ -44,24 +45,38 @@ def needs_build() -> bool:
 
 def build(force: bool = False, verbose: bool = False, out: Path | None = None, defines=()) -> Path:
     """out / defines: a variant build for A/B comparisons (e.g. ab/libmrlbm_X.so, -DNAME)."""
+    from concurrent.futures import ThreadPoolExecutor
+    import tempfile
+
     target = Path(out) if out else LIB
     if not force and not out and not needs_build():
         return LIB
     inc, lib = nccl_dirs()
     ncclso = "libnccl.so.2" if (lib / "libnccl.so.2").exists() else "libnccl.so"
     tmp = target.with_suffix(f".{os.getpid()}.tmp.so")
-    cmd = [nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "--expt-relaxed-constexpr",
-           "-Xcompiler", "-fPIC", "-shared", "-o", str(tmp), *map(str, SOURCES),
-           f"-I{ROOT / 'include'}", f"-I{inc}", f"-L{lib}", f"-l:{ncclso}",
-           "-Xlinker", f"-rpath,{lib}", *[f"-D{d}" for d in defines]]
+    common = [nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC",
+              f"-I{ROOT / 'include'}", f"-I{inc}", *[f"-D{d}" for d in defines]]
     if verbose:
-        cmd += ["-Xptxas", "-v"]
-    r = subprocess.run(cmd, capture_output=True, text=True)
-    if r.returncode != 0:
-        sys.stderr.write(r.stdout + r.stderr)
-        raise RuntimeError("nvcc failed building libmrlbm.so")
-    if verbose:
-        sys.stderr.write(r.stderr)
+        common += ["-Xptxas", "-v"]
+    with tempfile.TemporaryDirectory(prefix="mrlbm_build_") as td:
+        objs = [Path(td) / (src.stem + ".o") for src in SOURCES]
+
+        def compile_one(i):
+            return subprocess.run(common + ["-c", "-o", str(objs[i]), str(SOURCES[i])], capture_output=True, text=True)
+
+        with ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
+            results = list(ex.map(compile_one, range(len(SOURCES))))
+        for src, r in zip(SOURCES, results):
+            if r.returncode != 0:
+                sys.stderr.write(r.stdout + r.stderr)
+                raise RuntimeError(f"nvcc failed compiling {src.name}")
+            if verbose:
+                sys.stderr.write(f"== {src.name}\n" + r.stderr)
+        r = subprocess.run([nvcc(), *ARCH, "-shared", "-o", str(tmp), *map(str, objs), f"-L{lib}", f"-l:{ncclso}",
+                            "-lcuda", "-Xlinker", f"-rpath,{lib}"], capture_output=True, text=True)
+        if r.returncode != 0:
+            sys.stderr.write(r.stdout + r.stderr)
+            raise RuntimeError("nvcc failed linking libmrlbm.so")
     os.replace(tmp, target)
     return target
 

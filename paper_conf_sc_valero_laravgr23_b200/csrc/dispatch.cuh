@@ -1,0 +1,128 @@
+// dispatch.cuh -- template instances of the kernels behind a plain function
+// table (Variant / StVariant), so that each lattice compiles in its own
+// translation unit (var_d2q9.cu, var_d3q19.cu, var_d3q27.cu, var_st.cu) and the
+// host code (mrlbm.cu) selects one at mrlbm_create.
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+
+#include "../../include/mrlbm.h"
+#include "mrlbm_kernels.cuh"
+#include "st_kernels.cuh"
+
+namespace mrd {
+
+using mr::StepArgs;
+
+struct Variant {
+    int TA, TB, S, BW;
+    size_t smem;
+    void (*step)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t);
+    void (*step_push)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t); // P2P boundary layers (or null)
+    const void *kernel_fn_push;
+    void (*set)(const double *, void *, mr::GridArgs, cudaStream_t);
+    void (*get)(const void *, double *, mr::GridArgs, cudaStream_t);
+    void (*pops)(const void *, double *, mr::GridArgs, double, cudaStream_t);
+    void (*finite)(const void *, mr::GridArgs, int *, cudaStream_t);
+    void (*fd)(const mr::FdArgs &, long long, cudaStream_t);
+    const void *kernel_fn;
+};
+
+inline int grid_for(long long n) { return (int)std::min<long long>((n + 255) / 256, 148LL * 16); }
+
+template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB, bool WITH_PUSH = false> Variant make_variant()
+{
+    using L = mr::Lattice<LAT>;
+    using SM = mr::StepSmem<LAT, Real, TA, TB, S>;
+    Variant v;
+    v.TA = TA;
+    v.TB = TB;
+    v.S = S;
+    v.BW = SM::BW;
+    v.smem = SM::bytes;
+    v.kernel_fn = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB>;
+    v.step = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
+        mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB><<<grid, TA * TB, SM::bytes, st>>>(map, a);
+    };
+    v.step_push = nullptr;
+    v.kernel_fn_push = nullptr;
+    if constexpr (WITH_PUSH) {
+        v.kernel_fn_push = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true>;
+        v.step_push = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
+            mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true><<<grid, TA * TB, SM::bytes, st>>>(map, a);
+        };
+    }
+    v.set = [](const double *in, void *buf, mr::GridArgs g, cudaStream_t st) {
+        mr::set_moments_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
+            in, (Real *)buf, g);
+    };
+    v.get = [](const void *buf, double *out, mr::GridArgs g, cudaStream_t st) {
+        mr::get_moments_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
+            (const Real *)buf, out, g);
+    };
+    v.pops = [](const void *buf, double *out, mr::GridArgs g, double omega, cudaStream_t st) {
+        mr::populations_kernel<LAT, REC, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
+            (const Real *)buf, out, g, omega);
+    };
+    v.finite = [](const void *buf, mr::GridArgs g, int *flag, cudaStream_t st) {
+        mr::finite_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
+            (const Real *)buf, g, flag);
+    };
+    v.fd = [](const mr::FdArgs &a, long long nodes, cudaStream_t st) {
+        mr::fd_face_kernel<LAT, Real><<<grid_for(nodes), 256, 0, st>>>(a);
+    };
+    return v;
+}
+
+// ---- distribution representation (ST)
+struct StVariant {
+    int BX;
+    void (*step)(const mr::StArgs &, dim3, cudaStream_t);
+    void (*set)(const double *, void *, mr::StGrid, cudaStream_t);
+    void (*set_pops)(const double *, void *, mr::StGrid, cudaStream_t);
+    void (*get)(const void *, double *, mr::StGrid, cudaStream_t);
+    void (*pops)(const void *, double *, mr::StGrid, double, double, cudaStream_t);
+    void (*finite)(const void *, mr::StGrid, int *, cudaStream_t);
+    const void *kernel_fn;
+};
+
+template <int LAT, int COLL, typename Real> StVariant make_st()
+{
+    constexpr int BX = 128;
+    StVariant v;
+    v.BX = BX;
+    v.kernel_fn = (const void *)mr::st_step_kernel<LAT, COLL, Real, BX>;
+    v.step = [](const mr::StArgs &a, dim3 grid, cudaStream_t st) {
+        mr::st_step_kernel<LAT, COLL, Real, BX><<<grid, BX, 0, st>>>(a);
+    };
+    v.set = [](const double *in, void *buf, mr::StGrid g, cudaStream_t st) {
+        mr::st_set_moments_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(in, (Real *)buf, g);
+    };
+    v.set_pops = [](const double *in, void *buf, mr::StGrid g, cudaStream_t st) {
+        mr::st_set_populations_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(in, (Real *)buf, g);
+    };
+    v.get = [](const void *buf, double *out, mr::StGrid g, cudaStream_t st) {
+        mr::st_get_moments_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>((const Real *)buf, out, g);
+    };
+    v.pops = [](const void *buf, double *out, mr::StGrid g, double omega, double inv_tau, cudaStream_t st) {
+        mr::st_populations_kernel<LAT, COLL, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(
+            (const Real *)buf, out, g, omega, inv_tau);
+    };
+    v.finite = [](const void *buf, mr::StGrid g, int *flag, cudaStream_t st) {
+        mr::st_finite_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>((const Real *)buf, g, flag);
+    };
+    return v;
+}
+
+
+// per-lattice tables (one translation unit each)
+Variant pick_d2q9(bool rec, bool f32, int tile);
+Variant pick_d3q19(bool rec, bool f32, int tile);
+Variant pick_d3q27(bool rec, bool f32, int tile);
+StVariant select_st(int lat, int coll, int prec);
+// moments (eqs 1-3) of dense fp64 populations [Q][N] -> dense fp64 [M][N] (set_populations)
+void moments_of_populations(int lat, double *pops, double *mom, int nx, int rows, cudaStream_t st);
+
+} // namespace mrd

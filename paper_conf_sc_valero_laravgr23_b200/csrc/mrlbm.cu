@@ -23,8 +23,8 @@
 #include <vector>
 
 #include "../../include/mrlbm.h"
-#include "mrlbm_kernels.cuh"
-#include "st_kernels.cuh"
+#include "dispatch.cuh"
+#include "p2p_kernels.cuh"
 
 namespace {
 
@@ -51,161 +51,18 @@ mrlbm_status fail(mrlbm_status s, const std::string &msg)
 
 using mr::StepArgs;
 
-// ---------------------------------------------------------------- dispatch
-struct Variant {
-    int TA, TB, S, BW;
-    size_t smem;
-    void (*step)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t);
-    void (*step_push)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t); // P2P boundary layers (or null)
-    const void *kernel_fn_push;
-    void (*set)(const double *, void *, mr::GridArgs, cudaStream_t);
-    void (*get)(const void *, double *, mr::GridArgs, cudaStream_t);
-    void (*pops)(const void *, double *, mr::GridArgs, double, cudaStream_t);
-    void (*finite)(const void *, mr::GridArgs, int *, cudaStream_t);
-    void (*fd)(const mr::FdArgs &, long long, cudaStream_t);
-    const void *kernel_fn;
-};
-
-inline int grid_for(long long n) { return (int)std::min<long long>((n + 255) / 256, 148LL * 16); }
-
-template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB, bool WITH_PUSH = false> Variant make_variant()
-{
-    using L = mr::Lattice<LAT>;
-    using SM = mr::StepSmem<LAT, Real, TA, TB, S>;
-    Variant v;
-    v.TA = TA;
-    v.TB = TB;
-    v.S = S;
-    v.BW = SM::BW;
-    v.smem = SM::bytes;
-    v.kernel_fn = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB>;
-    v.step = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
-        mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB><<<grid, TA * TB, SM::bytes, st>>>(map, a);
-    };
-    v.step_push = nullptr;
-    v.kernel_fn_push = nullptr;
-    if constexpr (WITH_PUSH) {
-        v.kernel_fn_push = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true>;
-        v.step_push = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
-            mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true><<<grid, TA * TB, SM::bytes, st>>>(map, a);
-        };
-    }
-    v.set = [](const double *in, void *buf, mr::GridArgs g, cudaStream_t st) {
-        mr::set_moments_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
-            in, (Real *)buf, g);
-    };
-    v.get = [](const void *buf, double *out, mr::GridArgs g, cudaStream_t st) {
-        mr::get_moments_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
-            (const Real *)buf, out, g);
-    };
-    v.pops = [](const void *buf, double *out, mr::GridArgs g, double omega, cudaStream_t st) {
-        mr::populations_kernel<LAT, REC, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
-            (const Real *)buf, out, g, omega);
-    };
-    v.finite = [](const void *buf, mr::GridArgs g, int *flag, cudaStream_t st) {
-        mr::finite_kernel<L::M, Real><<<grid_for((long long)g.nA * g.nB * g.nC), 256, 0, st>>>(
-            (const Real *)buf, g, flag);
-    };
-    v.fd = [](const mr::FdArgs &a, long long nodes, cudaStream_t st) {
-        mr::fd_face_kernel<LAT, Real><<<grid_for(nodes), 256, 0, st>>>(a);
-    };
-    return v;
-}
-
-// Tile shapes: 2D one row of 128 threads (126 interior
-// nodes); 3D either 32 x 8 threads (30 x 6 interior, 2 CTAs/SM) or 32 x 16
-// threads (30 x 14 interior, 1 CTA/SM).  tile = 0: library default, 1: 32x8,
-// 2: 32x16 (MRLBM_TILE overrides, for tuning).
-template <int LAT, bool REC, typename Real> Variant pick(int tile)
-{
-    if constexpr (LAT == mr::LAT_D2Q9) {
-        // deeper TMA rings trade resident CTAs for bytes in flight (tuning: MRLBM_TILE)
-        if (tile == 1) return make_variant<LAT, REC, Real, 128, 1, 4, 4>();
-        if (tile == 2) return make_variant<LAT, REC, Real, 128, 1, 6, 4>();
-        if (tile == 3) return make_variant<LAT, REC, Real, 128, 1, 8, 3>();
-        return make_variant<LAT, REC, Real, 128, 1, 4, 5, true>();
-    } else {
-        constexpr bool f64 = sizeof(Real) == 8;
-        // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
-        constexpr bool small_only = LAT == mr::LAT_D3Q27 && f64;
-        if (tile == 0) tile = (LAT == mr::LAT_D3Q19 || small_only) ? 1 : 2;
-        // TMA ring depth: with the A-movers exchanged by shuffles the fp64 32x8
-        // tile fits three stages at two CTAs per SM; the 32x16 tile (one CTA
-        // per SM) takes four in fp32
-        // the library defaults also carry the P2P push instance
-        constexpr bool small_default = LAT == mr::LAT_D3Q19 || small_only;
-        if (tile == 1 || small_only) return make_variant<LAT, REC, Real, 32, 8, 3, 2, small_default>();
-        return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 4), 1, !small_default>();
-    }
-}
+using mrd::Variant;
+using mrd::StVariant;
+using mrd::select_st;
+using mrd::grid_for;
 
 Variant select_variant(int lat, int reg, int prec, int tile)
 {
     const bool R = reg == MRLBM_RECURSIVE;
     const bool F = prec == MRLBM_FP32;
-#define MR_SEL(LAT)                                                                                 \
-    if (R) return F ? pick<LAT, true, float>(tile) : pick<LAT, true, double>(tile);                 \
-    else return F ? pick<LAT, false, float>(tile) : pick<LAT, false, double>(tile);
-    if (lat == MRLBM_D2Q9) { MR_SEL(mr::LAT_D2Q9) }
-    if (lat == MRLBM_D3Q19) { MR_SEL(mr::LAT_D3Q19) }
-    MR_SEL(mr::LAT_D3Q27)
-#undef MR_SEL
-}
-
-// ---- distribution representation (ST) dispatch
-struct StVariant {
-    int BX;
-    void (*step)(const mr::StArgs &, dim3, cudaStream_t);
-    void (*set)(const double *, void *, mr::StGrid, cudaStream_t);
-    void (*set_pops)(const double *, void *, mr::StGrid, cudaStream_t);
-    void (*get)(const void *, double *, mr::StGrid, cudaStream_t);
-    void (*pops)(const void *, double *, mr::StGrid, double, double, cudaStream_t);
-    void (*finite)(const void *, mr::StGrid, int *, cudaStream_t);
-    const void *kernel_fn;
-};
-
-template <int LAT, int COLL, typename Real> StVariant make_st()
-{
-    constexpr int BX = 128;
-    StVariant v;
-    v.BX = BX;
-    v.kernel_fn = (const void *)mr::st_step_kernel<LAT, COLL, Real, BX>;
-    v.step = [](const mr::StArgs &a, dim3 grid, cudaStream_t st) {
-        mr::st_step_kernel<LAT, COLL, Real, BX><<<grid, BX, 0, st>>>(a);
-    };
-    v.set = [](const double *in, void *buf, mr::StGrid g, cudaStream_t st) {
-        mr::st_set_moments_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(in, (Real *)buf, g);
-    };
-    v.set_pops = [](const double *in, void *buf, mr::StGrid g, cudaStream_t st) {
-        mr::st_set_populations_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(in, (Real *)buf, g);
-    };
-    v.get = [](const void *buf, double *out, mr::StGrid g, cudaStream_t st) {
-        mr::st_get_moments_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>((const Real *)buf, out, g);
-    };
-    v.pops = [](const void *buf, double *out, mr::StGrid g, double omega, double inv_tau, cudaStream_t st) {
-        mr::st_populations_kernel<LAT, COLL, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>(
-            (const Real *)buf, out, g, omega, inv_tau);
-    };
-    v.finite = [](const void *buf, mr::StGrid g, int *flag, cudaStream_t st) {
-        mr::st_finite_kernel<LAT, Real><<<grid_for((long long)g.nx * g.ny * g.nz), 256, 0, st>>>((const Real *)buf, g, flag);
-    };
-    return v;
-}
-
-template <int LAT> StVariant pick_st(int coll, bool f32)
-{
-    if (coll == MRLBM_BGK) return f32 ? make_st<LAT, mr::COLL_BGK, float>() : make_st<LAT, mr::COLL_BGK, double>();
-    if (coll == MRLBM_RECURSIVE)
-        return f32 ? make_st<LAT, mr::COLL_RECURSIVE, float>() : make_st<LAT, mr::COLL_RECURSIVE, double>();
-    return f32 ? make_st<LAT, mr::COLL_PROJECTIVE, float>() : make_st<LAT, mr::COLL_PROJECTIVE, double>();
-}
-
-StVariant select_st(int lat, int coll, int prec)
-{
-    const bool F = prec == MRLBM_FP32;
-    if (lat == MRLBM_D2Q9) return pick_st<mr::LAT_D2Q9>(coll, F);
-    if (lat == MRLBM_D3Q19) return pick_st<mr::LAT_D3Q19>(coll, F);
-    return pick_st<mr::LAT_D3Q27>(coll, F);
+    if (lat == MRLBM_D2Q9) return mrd::pick_d2q9(R, F, tile);
+    if (lat == MRLBM_D3Q19) return mrd::pick_d3q19(R, F, tile);
+    return mrd::pick_d3q27(R, F, tile);
 }
 
 int env_int(const char *name, int dflt)
@@ -944,25 +801,8 @@ mrlbm_status mrlbm_set_populations(mrlbm_t h, const double *src, int64_t count)
     } else {
         // moments of f (eqs 1-3), computed by the ST moment kernel over a dense
         // [Q][N] view of the staging buffer, then stored as the MR state
-        mr::StGrid g;
-        g.nx = h->nA;
-        g.ny = h->nB * h->nC;
-        g.nz = 1;
-        g.pitch = h->nA;
-        g.plane = (long long)g.ny * g.pitch;
-        g.qstride = g.plane;
         double *mom = h->io + (size_t)h->Q * N;
-        const int lat = h->lattice;
-        if (lat == MRLBM_D2Q9) {
-            mr::st_set_populations_kernel<mr::LAT_D2Q9, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, h->io, g);
-            mr::st_get_moments_kernel<mr::LAT_D2Q9, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, mom, g);
-        } else if (lat == MRLBM_D3Q19) {
-            mr::st_set_populations_kernel<mr::LAT_D3Q19, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, h->io, g);
-            mr::st_get_moments_kernel<mr::LAT_D3Q19, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, mom, g);
-        } else {
-            mr::st_set_populations_kernel<mr::LAT_D3Q27, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, h->io, g);
-            mr::st_get_moments_kernel<mr::LAT_D3Q27, double><<<grid_for(N), 256, 0, h->stream>>>(h->io, mom, g);
-        }
+        mrd::moments_of_populations(h->lattice, h->io, mom, h->nA, h->nB * h->nC, h->stream);
         MR_CUDA(cudaGetLastError());
         h->var.set(mom, node0(h, h->cur), grid_args(h), h->stream);
         mrlbm_status ps = p2p_prologue(h);
@@ -1033,7 +873,7 @@ struct P2PBlob {
     uint64_t raw[3];                 // buf[0], buf[1], sync (same-process peers)
     cudaIpcMemHandle_t ipc[3];
 };
-constexpr uint32_t kP2PMagic = 0x4d52503250u; // "MRP2P"
+constexpr uint32_t kP2PMagic = 0x4d525032u; // "MRP2"
 static_assert(sizeof(P2PBlob) <= MRLBM_P2P_HANDLE_BYTES, "P2P handle blob too large");
 } // namespace
 

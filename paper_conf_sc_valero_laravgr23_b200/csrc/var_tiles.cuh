@@ -1,0 +1,35 @@
+// var_tiles.cuh -- tile shapes per lattice; included by
+// the per-lattice translation units only.
+#pragma once
+#include "dispatch.cuh"
+
+namespace mrd {
+
+// Tile shapes: 2D one row of 128 threads (126 interior
+// nodes); 3D either 32 x 8 threads (30 x 6 interior, 2 CTAs/SM) or 32 x 16
+// threads (30 x 14 interior, 1 CTA/SM).  tile = 0: library default, 1: 32x8,
+// 2: 32x16 (MRLBM_TILE overrides, for tuning).
+template <int LAT, bool REC, typename Real> Variant pick(int tile)
+{
+    if constexpr (LAT == mr::LAT_D2Q9) {
+        // deeper TMA rings trade resident CTAs for bytes in flight (tuning: MRLBM_TILE)
+        if (tile == 1) return make_variant<LAT, REC, Real, 128, 1, 4, 4>();
+        if (tile == 2) return make_variant<LAT, REC, Real, 128, 1, 6, 4>();
+        if (tile == 3) return make_variant<LAT, REC, Real, 128, 1, 8, 3>();
+        return make_variant<LAT, REC, Real, 128, 1, 4, 5, true>();
+    } else {
+        constexpr bool f64 = sizeof(Real) == 8;
+        // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
+        constexpr bool small_only = LAT == mr::LAT_D3Q27 && f64;
+        if (tile == 0) tile = (LAT == mr::LAT_D3Q19 || small_only) ? 1 : 2;
+        // TMA ring depth: with the A-movers exchanged by shuffles the fp64 32x8
+        // tile fits three stages at two CTAs per SM; the 32x16 tile (one CTA
+        // per SM) takes four in fp32
+        // the library defaults also carry the P2P push instance
+        constexpr bool small_default = LAT == mr::LAT_D3Q19 || small_only;
+        if (tile == 1 || small_only) return make_variant<LAT, REC, Real, 32, 8, 3, 2, small_default>();
+        return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 4), 1, !small_default>();
+    }
+}
+
+} // namespace mrd

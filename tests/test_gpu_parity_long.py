@@ -1,0 +1,113 @@
+"""GPU parity at the north-star horizon: every 3D variant (D3Q19 / D3Q27 x
+projective / recursive, fp64 and fp32) against the oracle after 1000 steps
+(BASELINE.json north_star: "after 1000 steps to max relative error 1e-11 in
+fp64 and 1e-4 in fp32"), on grids that span several tiles with ragged tails
+in x and y, and with the sweep axis cut into short segments (MRLBM_SEG=5:
+23 layers -> segments of 5,5,5,5,3, so every column crosses four segment
+seams, where a CTA starts / ends its sweep and re-reads a halo layer) as well
+as in the library's default segmentation.  Cases: fully periodic, lid-driven
+cavity (walls + moving wall), and open velocity / pressure faces on x and on
+y (regularized, R14) next to walls.
+
+The oracle runs once per physical case (module cache) and serves the fp64 /
+fp32 x segmentation variants of it."""
+import numpy as np
+import pytest
+
+from parity import assert_parity, group_errors, THREADS
+from paper_conf_sc_valero_laravgr23_b200 import inputs
+
+pytestmark = pytest.mark.gpu
+
+STEPS = 1000
+VARIANTS3 = [(l, r) for l in ("D3Q19", "D3Q27") for r in ("projective", "recursive")]
+_REF = {}
+
+
+def case(bc):
+    U = 0.04
+    if bc == "periodic":
+        return (33, 15, 23), 0.6, {}
+    if bc == "cavity":
+        return (33, 15, 23), 0.65, {"x-": {"kind": "wall"}, "x+": {"kind": "wall"}, "y-": {"kind": "wall"},
+                                    "y+": {"kind": "moving_wall", "u": [0.1, 0.0, 0.02]},
+                                    "z-": {"kind": "wall"}, "z+": {"kind": "moving_wall", "u": [0.0, -0.03, 0.0]}}
+    if bc == "open_x":
+        n = (31, 19, 23)
+        return n, 0.62, {"x-": {"kind": "velocity", "u_profile": inputs.channel3d_profile(n[1], n[2], U)},
+                         "x+": {"kind": "pressure", "rho": 1.0},
+                         "y-": {"kind": "wall"}, "y+": {"kind": "wall"}, "z-": {"kind": "wall"}, "z+": {"kind": "wall"}}
+    n = (31, 19, 23)
+    return n, 0.62, {"y-": {"kind": "velocity", "u": [0.0, U, 0.0]}, "y+": {"kind": "pressure", "rho": 0.999},
+                     "x-": {"kind": "wall"}, "x+": {"kind": "moving_wall", "u": [0.0, 0.0, 0.01]}}
+
+
+def reference(lat, reg, bc):
+    key = (lat, reg, bc)
+    if key not in _REF:
+        import oracle
+        (nx, ny, nz), tau, b = case(bc)
+        m0 = inputs.smooth_state(3, nx, ny, nz, U=0.04)
+        o = oracle.Oracle(lat, nx, ny, nz, tau, reg, b, threads=THREADS)
+        o.set_moments(m0)
+        o.step(STEPS)
+        _REF[key] = (m0, o.get_moments())
+    return _REF[key]
+
+
+def run_gpu(lat, reg, bc, precision, seg, monkeypatch):
+    from paper_conf_sc_valero_laravgr23_b200 import mrlbm
+    (nx, ny, nz), tau, b = case(bc)
+    m0, ref = reference(lat, reg, bc)
+    if seg:
+        monkeypatch.setenv("MRLBM_SEG", str(seg))
+    else:
+        monkeypatch.delenv("MRLBM_SEG", raising=False)
+    with mrlbm.Solver(lat, nx, ny, nz, tau, reg, b, precision=precision) as s:
+        cfg = s.kernel_config()
+        s.set_moments(m0)
+        s.step(STEPS)
+        got = s.get_moments()
+    if seg:
+        assert cfg["seg_len"] == seg and cfg["grid_y"] == -(-nz // seg), cfg
+    return group_errors(got, ref, 3)
+
+
+@pytest.mark.parametrize("seg", [0, 5], ids=["seg_default", "seg5"])
+@pytest.mark.parametrize("precision", ["fp64", "fp32"])
+@pytest.mark.parametrize("lat,reg", VARIANTS3)
+@pytest.mark.parametrize("bc", ["periodic", "cavity"])
+def test_3d_1000_steps(bc, lat, reg, precision, seg, monkeypatch):
+    errs = run_gpu(lat, reg, bc, precision, seg, monkeypatch)
+    assert_parity(errs, precision, f"{lat}-{reg} {bc} {precision} seg={seg or 'default'} 1000 steps")
+
+
+@pytest.mark.parametrize("seg", [0, 5], ids=["seg_default", "seg5"])
+@pytest.mark.parametrize("lat,reg", VARIANTS3)
+@pytest.mark.parametrize("bc", ["open_x", "open_y"])
+def test_3d_open_faces_1000_steps(bc, lat, reg, seg, monkeypatch):
+    errs = run_gpu(lat, reg, bc, "fp64", seg, monkeypatch)
+    assert_parity(errs, "fp64", f"{lat}-{reg} {bc} seg={seg or 'default'} 1000 steps")
+
+
+@pytest.mark.parametrize("lat,reg", [(l, r) for l in ("D2Q9",) for r in ("projective", "recursive")])
+def test_2d_short_segments_1000_steps(lat, reg, monkeypatch):
+    """2D with MRLBM_SEG=5: 67 rows -> 14 segments (ragged last one)."""
+    from paper_conf_sc_valero_laravgr23_b200 import mrlbm
+    import oracle
+    nx, ny = 131, 67
+    b = {"x-": {"kind": "wall"}, "x+": {"kind": "wall"}, "y-": {"kind": "wall"},
+         "y+": {"kind": "moving_wall", "u": [0.1, 0.0, 0.0]}}
+    m0 = inputs.smooth_state(2, nx, ny, 1, U=0.05)
+    o = oracle.Oracle(lat, nx, ny, 1, 0.65, reg, b, threads=THREADS)
+    o.set_moments(m0)
+    o.step(STEPS)
+    ref = o.get_moments()
+    monkeypatch.setenv("MRLBM_SEG", "5")
+    for precision in ("fp64", "fp32"):
+        with mrlbm.Solver(lat, nx, ny, 1, 0.65, reg, b, precision=precision) as s:
+            assert s.kernel_config()["grid_y"] == 14
+            s.set_moments(m0)
+            s.step(STEPS)
+            got = s.get_moments()
+        assert_parity(group_errors(got, ref, 2), precision, f"{lat}-{reg} seg5 {precision}")
