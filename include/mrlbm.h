@@ -174,14 +174,27 @@ mrlbm_status mrlbm_get_populations(mrlbm_t h, double *dst, int64_t count);
 mrlbm_status mrlbm_set_populations(mrlbm_t h, const double *src, int64_t count);
 
 /* Device-side variants for zero-copy I/O: dst/src are DEVICE pointers to fp64
- * arrays in the host layout above; enqueued on the handle's stream. */
+ * arrays in the host layout above.  The copy runs on the handle's stream and
+ * the call returns after it completed (synchronous, like the host variants):
+ * the caller must have finished writing src (e.g. synchronised the stream that
+ * produced it) and may reuse or free the buffer as soon as the call returns.
+ * On a P2P-transport handle the set variants require mrlbm_p2p_connect first
+ * (MRLBM_ERR_INVALID_ARGUMENT otherwise: the neighbours' ghost planes could
+ * not be filled). */
 mrlbm_status mrlbm_set_moments_device(mrlbm_t h, const double *src_dev, int64_t count);
 mrlbm_status mrlbm_get_moments_device(mrlbm_t h, double *dst_dev, int64_t count);
 
-/* Wait for all enqueued work. */
+/* Wait for all enqueued work.  P2P transport: MRLBM_ERR_CUDA if a halo wait
+ * timed out (a neighbour stopped); the handle then refuses further steps. */
 mrlbm_status mrlbm_sync(mrlbm_t h);
 
-/* Scan the state for non-finite values (debug aid); MRLBM_ERR_NUMERICAL if any. */
+/* Halo transport of a handle: *transport = 0 single rank, 1 NCCL, 2 P2P,
+ * 3 slab group; for NCCL *comm_nranks / *comm_rank are what the communicator
+ * reports (ncclCommCount / ncclCommUserRank), else nranks / rank. */
+mrlbm_status mrlbm_comm_info(mrlbm_t h, int *transport, int *comm_nranks, int *comm_rank);
+
+/* Scan the state for non-finite values (debug aid); MRLBM_ERR_NUMERICAL if any
+ * (MRLBM_ERR_CUDA first if a P2P halo wait timed out). */
 mrlbm_status mrlbm_check_finite(mrlbm_t h);
 
 /* Sizes: M, Q, local march extent, its global offset, device bytes held. */

@@ -33,12 +33,14 @@ class Config:
     def nodes(self):
         return self.nx * self.ny * (1 if self.D == 2 else self.nz)
 
-    def initial_moments(self, seed=inputs.SEED):
+    def initial_moments(self, seed=inputs.SEED, lo=0, hi=None):
+        """ABI moments of the initial state; lo, hi: only layers [lo, hi) of the
+        slowest axis (z in 3D, y in 2D) -- one rank's slab"""
         if self.init == "poiseuille":
-            return inputs.poiseuille_state(self.nx, self.ny, self.U, self.tau)
+            return inputs.poiseuille_state(self.nx, self.ny, self.U, self.tau)[:, lo:hi]
         if self.init == "taylor_green_3d":
-            return inputs.taylor_green_3d(self.nx, self.U, self.tau)
-        return inputs.perturbed_rest(self.D, self.nx, self.ny, self.nz, self.U, seed)
+            return inputs.taylor_green_3d(self.nx, self.U, self.tau)[:, lo:hi]
+        return inputs.perturbed_rest(self.D, self.nx, self.ny, self.nz, self.U, seed, lo=lo, hi=hi)
 
 
 def _walls(D, lid_face=None, U=0.0):

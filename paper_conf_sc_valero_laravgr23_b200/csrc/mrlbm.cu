@@ -156,8 +156,9 @@ mr::GridArgs grid_args(const mrlbm_ctx *h)
     return g;
 }
 
-// launch the fused kernel over owned layers [cb, ce) reading buf[src]
-void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st, bool push = false)
+// launch the fused kernel over owned layers [cb, ce) (and, if ce2 > cb2, also
+// over [cb2, ce2) in the same launch) reading buf[src]
+void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st, bool push = false, int cb2 = 0, int ce2 = 0)
 {
     if (ce <= cb) return;
     StepArgs a = h->base;
@@ -172,11 +173,24 @@ void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st, bool p
     a.c_end = ce;
     const int span = ce - cb;
     a.seg_len = std::min(h->seg_len, span);
-    const int nseg = (span + a.seg_len - 1) / a.seg_len;
+    a.nseg1 = (span + a.seg_len - 1) / a.seg_len;
+    int nseg = a.nseg1;
+    if (ce2 > cb2) { // second range: segments nseg1.. of the grid (same segment length)
+        a.c2_begin = cb2;
+        a.c2_end = ce2;
+        nseg += (ce2 - cb2 + a.seg_len - 1) / a.seg_len;
+    }
     dim3 grid(h->tilesA * h->tilesB, nseg);
     if (push) h->var.step_push(h->tmap[src], a, grid, st);
     else h->var.step(h->tmap[src], a, grid, st);
     h->kernels++;
+}
+
+// the slab's first and last layer (they read the ghost planes) in one launch
+void launch_boundary(mrlbm_ctx *h, int src, cudaStream_t st, bool push)
+{
+    if (h->nC == 1) launch_range(h, src, 0, 1, st, push);
+    else launch_range(h, src, 0, 1, st, push, h->nC - 1, h->nC);
 }
 
 mrlbm_status enqueue_one_step(mrlbm_ctx *h, cudaStream_t st)
@@ -197,9 +211,8 @@ mrlbm_status enqueue_one_step(mrlbm_ctx *h, cudaStream_t st)
         if (!h->p2p_connected) return fail(MRLBM_ERR_INVALID_ARGUMENT, "P2P transport: mrlbm_p2p_connect first");
         launch_range(h, src, 1, h->nC - 1, st);
         mr::p2p_wait_kernel<<<1, 1, 0, st>>>(h->sync, h->nb_lo >= 0, h->nb_hi >= 0, h->p2p_err);
-        launch_range(h, src, 0, 1, st, true);
-        launch_range(h, src, h->nC - 1, h->nC, st, true);
-        mr::p2p_signal_kernel<<<1, 1, 0, st>>>(h->sync, h->peer_sync_lo, h->peer_sync_hi);
+        launch_boundary(h, src, st, true); // layers 0 and nC-1 in one launch, pushes fused
+        mr::p2p_signal_kernel<<<1, 1, 0, st>>>(h->sync, h->peer_sync_lo, h->peer_sync_hi, h->p2p_err);
         h->kernels += 2;
     } else if (h->nranks == 1) {
         launch_range(h, src, 0, h->nC, st);
@@ -232,16 +245,19 @@ mrlbm_status enqueue_one_step(mrlbm_ctx *h, cudaStream_t st)
         const ncclDataType_t dt = h->prec == MRLBM_FP32 ? ncclFloat32 : ncclFloat64;
         const size_t cnt = (size_t)h->pstride;
         MR_NCCL(ncclGroupStart());
-        if (h->nb_hi >= 0) MR_NCCL(ncclSend(base + plane * h->nC, cnt, dt, h->nb_hi, h->comm, h->comm_stream));
-        if (h->nb_lo >= 0) MR_NCCL(ncclSend(base + plane * 1, cnt, dt, h->nb_lo, h->comm, h->comm_stream));
-        if (h->nb_lo >= 0) MR_NCCL(ncclRecv(base, cnt, dt, h->nb_lo, h->comm, h->comm_stream));
-        if (h->nb_hi >= 0) MR_NCCL(ncclRecv(base + plane * (h->nC + 1), cnt, dt, h->nb_hi, h->comm, h->comm_stream));
-        MR_NCCL(ncclGroupEnd());
+        ncclResult_t r = ncclSuccess;
+        if (r == ncclSuccess && h->nb_hi >= 0) r = ncclSend(base + plane * h->nC, cnt, dt, h->nb_hi, h->comm, h->comm_stream);
+        if (r == ncclSuccess && h->nb_lo >= 0) r = ncclSend(base + plane * 1, cnt, dt, h->nb_lo, h->comm, h->comm_stream);
+        if (r == ncclSuccess && h->nb_lo >= 0) r = ncclRecv(base, cnt, dt, h->nb_lo, h->comm, h->comm_stream);
+        if (r == ncclSuccess && h->nb_hi >= 0)
+            r = ncclRecv(base + plane * (h->nC + 1), cnt, dt, h->nb_hi, h->comm, h->comm_stream);
+        const ncclResult_t re = ncclGroupEnd(); // always close the group, also on error
+        if (r != ncclSuccess) return fail(MRLBM_ERR_NCCL, std::string("ncclSend/ncclRecv: ") + ncclGetErrorString(r));
+        if (re != ncclSuccess) return fail(MRLBM_ERR_NCCL, std::string("ncclGroupEnd: ") + ncclGetErrorString(re));
         MR_CUDA(cudaEventRecord(h->ev_comm, h->comm_stream));
         launch_range(h, src, 1, h->nC - 1, st);
         MR_CUDA(cudaStreamWaitEvent(st, h->ev_comm, 0));
-        launch_range(h, src, 0, 1, st);
-        launch_range(h, src, h->nC - 1, h->nC, st);
+        launch_boundary(h, src, st, false); // layers 0 and nC-1 in one launch
     }
     h->cur ^= 1;
     MR_CUDA(cudaGetLastError());
@@ -266,7 +282,9 @@ mrlbm_status ensure_io(mrlbm_ctx *h, size_t bytes)
 // neighbours' ghost planes of the current buffer (ordered like a step's push)
 mrlbm_status p2p_prologue(mrlbm_ctx *h)
 {
-    if (!h->p2p || !h->p2p_connected) return MRLBM_OK;
+    if (!h->p2p) return MRLBM_OK;
+    if (!h->p2p_connected) // the neighbours' ghost planes cannot be filled: refuse (header)
+        return fail(MRLBM_ERR_INVALID_ARGUMENT, "P2P transport: mrlbm_p2p_connect before setting the state");
     const int b = h->cur;
     char *base = (char *)h->buf[b];
     const size_t plane = (size_t)h->pstride * h->wbytes;
@@ -279,9 +297,18 @@ mrlbm_status p2p_prologue(mrlbm_ctx *h)
         mr::p2p_push_planes_kernel<double><<<grid_for(h->pstride), 256, 0, h->stream>>>(
             (const double *)(base + plane), (const double *)(base + plane * h->nC), (double *)h->peer_plane_lo[b],
             (double *)h->peer_plane_hi[b], h->pstride);
-    mr::p2p_signal_kernel<<<1, 1, 0, h->stream>>>(h->sync, h->peer_sync_lo, h->peer_sync_hi);
+    mr::p2p_signal_kernel<<<1, 1, 0, h->stream>>>(h->sync, h->peer_sync_lo, h->peer_sync_hi, h->p2p_err);
     MR_CUDA(cudaGetLastError());
     return MRLBM_OK;
+}
+
+// P2P: a halo wait that timed out poisons the handle (its ghosts are stale)
+mrlbm_status p2p_check(mrlbm_ctx *h)
+{
+    if (!h->p2p_err) return MRLBM_OK;
+    int e = 0;
+    MR_CUDA(cudaMemcpy(&e, h->p2p_err, sizeof(int), cudaMemcpyDeviceToHost));
+    return e ? fail(MRLBM_ERR_CUDA, "P2P transport: a neighbour stopped (halo wait timed out)") : MRLBM_OK;
 }
 
 bool is_wall(int k) { return k == MRLBM_WALL || k == MRLBM_MOVING_WALL; }
@@ -731,10 +758,15 @@ mrlbm_status mrlbm_set_moments_device(mrlbm_t h, const double *src_dev, int64_t 
 {
     if (!h || !src_dev) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
     if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
+    if (h->p2p && !h->p2p_connected)
+        return fail(MRLBM_ERR_INVALID_ARGUMENT, "P2P transport: mrlbm_p2p_connect before setting the state");
     if (h->repr == MRLBM_DISTRIBUTIONS) h->sv.set(src_dev, h->buf[h->cur], h->st_grid, h->stream);
     else h->var.set(src_dev, node0(h, h->cur), grid_args(h), h->stream);
     MR_CUDA(cudaGetLastError());
-    return p2p_prologue(h);
+    mrlbm_status s = p2p_prologue(h);
+    if (s) return s;
+    MR_CUDA(cudaStreamSynchronize(h->stream)); // synchronous: src may be reused on return
+    return MRLBM_OK;
 }
 
 mrlbm_status mrlbm_get_moments_device(mrlbm_t h, double *dst_dev, int64_t count)
@@ -744,7 +776,8 @@ mrlbm_status mrlbm_get_moments_device(mrlbm_t h, double *dst_dev, int64_t count)
     if (h->repr == MRLBM_DISTRIBUTIONS) h->sv.get(h->buf[h->cur], dst_dev, h->st_grid, h->stream);
     else h->var.get(node0(h, h->cur), dst_dev, grid_args(h), h->stream);
     MR_CUDA(cudaGetLastError());
-    return MRLBM_OK;
+    MR_CUDA(cudaStreamSynchronize(h->stream)); // synchronous: dst is complete on return
+    return p2p_check(h);
 }
 
 mrlbm_status mrlbm_set_moments(mrlbm_t h, const double *src, int64_t count)
@@ -791,6 +824,8 @@ mrlbm_status mrlbm_set_populations(mrlbm_t h, const double *src, int64_t count)
 {
     if (!h || !src) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
     if (h->group_mode) return fail(MRLBM_ERR_UNSUPPORTED, "set_populations on a slab-group handle");
+    if (h->p2p && !h->p2p_connected)
+        return fail(MRLBM_ERR_INVALID_ARGUMENT, "P2P transport: mrlbm_p2p_connect before setting the state");
     const int64_t N = local_nodes(h);
     if (count != (int64_t)h->Q * N) return fail(MRLBM_ERR_BUFFER_SIZE, "count != Q * N_local");
     mrlbm_status s = ensure_io(h, (size_t)(h->Q + h->M) * N * sizeof(double));
@@ -856,12 +891,7 @@ mrlbm_status mrlbm_sync(mrlbm_t h)
     if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
     MR_CUDA(cudaStreamSynchronize(h->stream));
     if (h->comm_stream) MR_CUDA(cudaStreamSynchronize(h->comm_stream));
-    if (h->p2p_err) {
-        int e = 0;
-        MR_CUDA(cudaMemcpy(&e, h->p2p_err, sizeof(int), cudaMemcpyDeviceToHost));
-        if (e) return fail(MRLBM_ERR_CUDA, "P2P transport: a neighbour stopped (wait timed out)");
-    }
-    return MRLBM_OK;
+    return p2p_check(h);
 }
 
 // ---------------------------------------------------------------- P2P transport setup
@@ -959,6 +989,9 @@ mrlbm_status mrlbm_p2p_connect(mrlbm_t h, const void *blob_lo, const void *blob_
 mrlbm_status mrlbm_check_finite(mrlbm_t h)
 {
     if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
+    MR_CUDA(cudaStreamSynchronize(h->stream));
+    mrlbm_status ps = p2p_check(h);
+    if (ps) return ps;
     MR_CUDA(cudaMemsetAsync(h->flag, 0, sizeof(int), h->stream));
     if (h->repr == MRLBM_DISTRIBUTIONS) h->sv.finite(h->buf[h->cur], h->st_grid, h->flag, h->stream);
     else h->var.finite(node0(h, h->cur), grid_args(h), h->flag, h->stream);
@@ -976,6 +1009,21 @@ mrlbm_status mrlbm_query(mrlbm_t h, int64_t *M, int64_t *Q, int64_t *n_local, in
     if (n_local) *n_local = h->nC;
     if (offset) *offset = h->coff;
     if (bytes) *bytes = (int64_t)(2 * h->buf_bytes);
+    return MRLBM_OK;
+}
+
+mrlbm_status mrlbm_comm_info(mrlbm_t h, int *transport, int *comm_nranks, int *comm_rank)
+{
+    if (!h) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null handle");
+    int t = h->nranks == 1 ? 0 : (h->p2p ? 2 : (h->group_mode ? 3 : 1));
+    int n = h->nranks, r = h->rank;
+    if (h->comm) {
+        MR_NCCL(ncclCommCount(h->comm, &n));
+        MR_NCCL(ncclCommUserRank(h->comm, &r));
+    }
+    if (transport) *transport = t;
+    if (comm_nranks) *comm_nranks = n;
+    if (comm_rank) *comm_rank = r;
     return MRLBM_OK;
 }
 
@@ -1036,8 +1084,7 @@ mrlbm_status mrlbm_step_group(mrlbm_t *hs, int n_handles, int64_t n)
         for (int r = 0; r < n_handles; r++) {
             mrlbm_ctx *h = hs[r];
             launch_range(h, h->cur, 1, h->nC - 1, st);
-            launch_range(h, h->cur, 0, 1, st);
-            launch_range(h, h->cur, h->nC - 1, h->nC, st);
+            launch_boundary(h, h->cur, st, false);
         }
         for (int r = 0; r < n_handles; r++) hs[r]->cur ^= 1;
         MR_CUDA(cudaGetLastError());

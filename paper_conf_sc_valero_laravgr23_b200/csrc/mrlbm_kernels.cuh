@@ -38,8 +38,10 @@ struct StepArgs {
     int pitch;              // elements per A-row
     long long mstride;      // elements between moment planes = nB * pitch
     long long pstride;      // elements between layers         = M * nB * pitch
-    int c_begin, c_end;     // owned layers updated by this launch
+    int c_begin, c_end;     // owned layers updated by this launch (segments 0 .. nseg1-1 of grid.y)
     int seg_len;            // layers per CTA segment
+    int nseg1;              // segments of the first range; grid.y beyond it covers [c2_begin, c2_end)
+    int c2_begin, c2_end;   // optional second range (a slab's first and last layer in one launch)
     int tilesA;             // tiles along A (grid.x = tilesA * tilesB)
     int lo_nb, hi_nb;       // 1 if layer -1 / nC exists (periodic wrap or ghost plane)
     int wrapC;              // 1: layer c lives in plane wrap(c)+1 (single-rank periodic C)
@@ -636,8 +638,9 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     const int a = a0 + tx, b = b0 + ty;
     const int nA = p.nA, nB = p.nB, nC = p.nC;
 
-    const int c0 = p.c_begin + blockIdx.y * p.seg_len;
-    const int c1 = min(c0 + p.seg_len, p.c_end);
+    const bool second = (int)blockIdx.y >= p.nseg1;
+    const int c0 = second ? p.c2_begin + ((int)blockIdx.y - p.nseg1) * p.seg_len : p.c_begin + blockIdx.y * p.seg_len;
+    const int c1 = min(c0 + p.seg_len, second ? p.c2_end : p.c_end);
     if (c0 >= c1) return;
     const int boxA = ((a0 + p.padA) / SM::AL) * SM::AL; // aligned TMA box origin (a0 + padA >= 0)
     const int offA = a0 + p.padA - boxA;                  // window column 0 inside the box

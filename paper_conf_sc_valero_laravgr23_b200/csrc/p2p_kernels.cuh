@@ -32,6 +32,7 @@ __device__ __forceinline__ unsigned long long globaltimer_ns()
 
 __global__ void p2p_wait_kernel(unsigned long long *sync, int need_lo, int need_hi, int *err)
 {
+    if (*(volatile int *)err) return; // already failed: no further 30 s waits (mrlbm_sync reports it)
     const unsigned long long target = sync[0];
     const unsigned long long t0 = globaltimer_ns();
     while ((need_lo && ld_acquire_sys(&sync[1]) < target) || (need_hi && ld_acquire_sys(&sync[2]) < target)) {
@@ -43,8 +44,12 @@ __global__ void p2p_wait_kernel(unsigned long long *sync, int need_lo, int need_
     }
 }
 
-__global__ void p2p_signal_kernel(unsigned long long *sync, unsigned long long *lo_sync, unsigned long long *hi_sync)
+__global__ void p2p_signal_kernel(unsigned long long *sync, unsigned long long *lo_sync, unsigned long long *hi_sync,
+                                  const int *err)
 {
+    // after a timed-out wait this rank's boundary layers used stale ghosts: stop
+    // signalling, so the neighbours time out (and report) instead of reading them
+    if (*(volatile const int *)err) return;
     __threadfence_system();
     const unsigned long long c = sync[0] + 1;
     sync[0] = c;

@@ -29,18 +29,45 @@ def n_moments(D: int) -> int:
     return 6 if D == 2 else 10
 
 
+class _Modes:
+    """Sum of nmodes random-phase low-wavenumber Fourier modes on a periodic
+    grid (slowest axis first).  The random parameters are drawn at
+    construction (phase, then one wavenumber 1..3 per axis, per mode); the
+    field is evaluated on any range [lo, hi) of the slowest axis, so a slab
+    of a multi-GPU decomposition gets exactly its part of the global field
+    without building the rest."""
+
+    def __init__(self, rng, grid, amp, nmodes=4):
+        self.grid, self.amp, self.nmodes = tuple(grid), amp, nmodes
+        self.params = []
+        for _ in range(nmodes):
+            ph = rng.uniform(0, 2 * np.pi)
+            ks = [int(rng.integers(1, 4)) for _ in grid]
+            self.params.append((ph, ks))
+
+    def eval(self, lo=0, hi=None):
+        hi = self.grid[0] if hi is None else hi
+        shape = (hi - lo,) + self.grid[1:]
+        # cos(ph + sum_a 2 pi k_a x_a / n_a) = Re(P(x_0..x_{D-2}) F(x_{D-1})) with
+        # per-axis phase factors: the mode sum is one small real matrix product
+        # [Re P | -Im P] @ [Re F ; Im F] (no full-size argument or cos array)
+        L = np.empty((int(np.prod(shape[:-1])), 2 * self.nmodes))
+        R = np.empty((2 * self.nmodes, shape[-1]))
+        for m, (ph, ks) in enumerate(self.params):
+            P = np.exp(1j * ph) * np.ones(shape[:-1], dtype=complex)
+            for a, (k, n) in enumerate(zip(ks[:-1], self.grid[:-1])):
+                idx = np.arange(lo, hi) if a == 0 else np.arange(n)
+                f = np.exp(2j * np.pi * k * idx / n)
+                P = P * f.reshape([-1 if b == a else 1 for b in range(len(shape) - 1)])
+            F = np.exp(2j * np.pi * ks[-1] * np.arange(shape[-1]) / self.grid[-1])
+            L[:, 2 * m], L[:, 2 * m + 1] = P.real.reshape(-1), -P.imag.reshape(-1)
+            R[2 * m], R[2 * m + 1] = F.real, F.imag
+        return (self.amp / self.nmodes) * (L @ R).reshape(shape)
+
+
 def _modes(rng, grid, amp, nmodes=4):
     """Sum of nmodes random-phase low-wavenumber Fourier modes on a periodic grid."""
-    axes = np.meshgrid(*[np.arange(n) for n in grid], indexing="ij")
-    out = np.zeros(grid)
-    for _ in range(nmodes):
-        ph = rng.uniform(0, 2 * np.pi)
-        arg = ph
-        for ax, n in zip(axes, grid):
-            k = rng.integers(1, 4)
-            arg = arg + 2 * np.pi * k * ax / n
-        out += np.cos(arg)
-    return amp * out / nmodes
+    return _Modes(rng, grid, amp, nmodes).eval()
 
 
 def pack(rho, u, Pi) -> np.ndarray:
@@ -56,31 +83,61 @@ def _grid(D, nx, ny, nz):
     return (ny, nx) if D == 2 else (nz, ny, nx)
 
 
-def perturbed_rest(D, nx, ny, nz=1, U=0.05, seed=SEED, pi_neq=True):
-    """Rest state (rho=1, u=0) plus seeded random-phase perturbations."""
+def perturbed_rest(D, nx, ny, nz=1, U=0.05, seed=SEED, pi_neq=True, lo=0, hi=None, chunk=16):
+    """Rest state (rho=1, u=0) plus seeded random-phase perturbations.
+    lo, hi: range of the slowest axis (z in 3D, y in 2D) to return -- a slab
+    of the global field, generated in chunks of `chunk` planes straight into
+    the output (bench: one 1024 x 1024 x 128 slab per GPU)."""
     rng = np.random.default_rng(seed)
     g = _grid(D, nx, ny, nz)
-    rho = 1.0 + _modes(rng, g, 1e-3)
-    u = [_modes(rng, g, 1e-3 * U) for _ in range(D)]
-    Pi = [[None] * D for _ in range(D)]
+    hi = g[0] if hi is None else hi
+    m_rho = _Modes(rng, g, 1e-3)
+    m_u = [_Modes(rng, g, 1e-3 * U) for _ in range(D)]
+    m_pi = {}
     for a in range(D):
         for b in range(a, D):
-            v = rho * u[a] * u[b]
+            m_pi[(a, b)] = _Modes(rng, g, 1e-4 * U * U) if pi_neq else None
+    out = np.empty((n_moments(D), hi - lo) + g[1:])
+    for c0 in range(lo, hi, chunk):
+        c1 = min(hi, c0 + chunk)
+        o = out[:, c0 - lo:c1 - lo]
+        rho = o[0]
+        rho[...] = m_rho.eval(c0, c1)
+        rho += 1.0
+        u = []
+        for a in range(D):
+            o[1 + a] = m_u[a].eval(c0, c1)
+            u.append(o[1 + a])
+        for (a, b), slot in _pi_slots(D).items():
+            v = o[slot]
             if pi_neq:
-                v = v + _modes(rng, g, 1e-4 * U * U)
-            Pi[a][b] = Pi[b][a] = v
-    return pack(rho, u, Pi)
+                v[...] = m_pi[(a, b)].eval(c0, c1)
+                v += rho * u[a] * u[b]
+            else:
+                v[...] = rho * u[a] * u[b]
+    return out
 
 
-def smooth_state(D, nx, ny, nz=1, U=0.05, seed=SEED):
+def _pi_slots(D):
+    """ABI slot of Pi_ab (a <= b), in the generation order of perturbed_rest"""
+    if D == 2:
+        return {(0, 0): 3, (0, 1): 5, (1, 1): 4}
+    return {(0, 0): 4, (0, 1): 7, (0, 2): 8, (1, 1): 5, (1, 2): 9, (2, 2): 6}
+
+
+def smooth_state(D, nx, ny, nz=1, U=0.05, seed=SEED, mean_u=None):
     """Smooth seeded flow of order U: 4 random-phase modes on every moment
     (rho: 1e-2, u: U, Pi^neq: 1e-3 U) -- parity tests (every Hermite term
     and every velocity component is O(U), so the per-group metric is not
-    dominated by absolute rounding of near-zero fields)."""
+    dominated by absolute rounding of near-zero fields).  mean_u: a uniform
+    velocity added to u (periodic runs long enough for the modes to decay
+    viscously keep an O(U) field)."""
     rng = np.random.default_rng(seed)
     g = _grid(D, nx, ny, nz)
     rho = 1.0 + _modes(rng, g, 1e-2)
     u = [_modes(rng, g, U) for _ in range(D)]
+    if mean_u is not None:
+        u = [u[a] + mean_u[a] for a in range(D)]
     Pi = [[None] * D for _ in range(D)]
     for a in range(D):
         for b in range(a, D):

@@ -40,7 +40,7 @@ API = ("mrlbm_default_options", "mrlbm_create", "mrlbm_set_moments", "mrlbm_step
        "mrlbm_get_populations", "mrlbm_set_moments_device", "mrlbm_get_moments_device", "mrlbm_sync",
        "mrlbm_check_finite", "mrlbm_query", "mrlbm_launch_count", "mrlbm_time_steps", "mrlbm_destroy",
        "mrlbm_status_string", "mrlbm_last_error", "mrlbm_nccl_unique_id", "mrlbm_set_populations",
-       "mrlbm_p2p_handle", "mrlbm_p2p_connect")
+       "mrlbm_p2p_handle", "mrlbm_p2p_connect", "mrlbm_comm_info")
 HOST_HELPERS = ("mrlbm_partition", "mrlbm_validate", "mrlbm_validate_repr", "mrlbm_kernel_config", "mrlbm_step_group")
 
 
@@ -94,6 +94,7 @@ def _load():
         "mrlbm_step_group": (ctypes.c_int, [ctypes.POINTER(vp), ctypes.c_int, i64]),
         "mrlbm_p2p_handle": (ctypes.c_int, [vp, vp]),
         "mrlbm_p2p_connect": (ctypes.c_int, [vp, vp, vp]),
+        "mrlbm_comm_info": (ctypes.c_int, [vp, ip, ip, ip]),
     }
     for name, (res, args) in sig.items():
         if not hasattr(L, name) and os.environ.get("MRLBM_LIB"):
@@ -249,13 +250,20 @@ class Solver:
                "mrlbm_set_populations")
 
     # ---- device I/O (torch fp64 CUDA tensors in the ABI layout)
+    # The library copies on its own stream and returns when the copy is done;
+    # the tensor's producer on torch's current stream must be finished first.
     def set_moments_device(self, t):
-        assert t.is_contiguous() and str(t.dtype) == "torch.float64"
+        import torch
+        assert t.is_contiguous() and t.dtype == torch.float64 and t.is_cuda
+        torch.cuda.current_stream(t.device).synchronize()
         _check(lib.mrlbm_set_moments_device(self._h, ctypes.c_void_p(t.data_ptr()), t.numel()),
                "mrlbm_set_moments_device")
 
     def get_moments_device(self, t):
-        assert t.is_contiguous() and str(t.dtype) == "torch.float64"
+        import torch
+        assert t.is_contiguous() and t.dtype == torch.float64 and t.is_cuda
+        # t must not be in use by torch's stream while the library writes it
+        torch.cuda.current_stream(t.device).synchronize()
         _check(lib.mrlbm_get_moments_device(self._h, ctypes.c_void_p(t.data_ptr()), t.numel()),
                "mrlbm_get_moments_device")
 
@@ -282,6 +290,13 @@ class Solver:
 
     def check_finite(self):
         _check(lib.mrlbm_check_finite(self._h), "mrlbm_check_finite")
+
+    def comm_info(self) -> dict:
+        """halo transport and the communicator's own view of the rank count"""
+        t, n, r = ctypes.c_int(), ctypes.c_int(), ctypes.c_int()
+        _check(lib.mrlbm_comm_info(self._h, ctypes.byref(t), ctypes.byref(n), ctypes.byref(r)), "mrlbm_comm_info")
+        return {"transport": ["single", "nccl", "p2p", "slab_group"][t.value], "comm_nranks": n.value,
+                "comm_rank": r.value}
 
     def launch_count(self) -> int:
         k = ctypes.c_int64()

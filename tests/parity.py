@@ -25,6 +25,11 @@ def group_errors(gpu, ref, D):
     return out
 
 
+def group_scales(ref, D):
+    """max|oracle| per group (the denominators of group_errors), for messages"""
+    return {g: float(np.abs(ref[idx]).max()) for g, idx in groups(D).items()}
+
+
 def run_pair(lat, reg, nx, ny, nz, tau, boundary, m0, steps, precision="fp64"):
     import oracle
     from paper_conf_sc_valero_laravgr23_b200 import mrlbm

@@ -64,6 +64,25 @@ def test_p2p_in_process_bitwise(case, P):
     assert np.array_equal(got, ref), f"max diff {np.abs(got - ref).max()}"
 
 
+def test_p2p_set_before_connect_is_refused():
+    """The neighbours' ghost planes can only be filled once connected: setting
+    the state of a P2P handle before mrlbm_p2p_connect is an error, not a
+    silent zero halo."""
+    from paper_conf_sc_valero_laravgr23_b200 import mrlbm
+    nx, ny, nz = 19, 13, 12
+    m0 = inputs.smooth_state(3, nx, ny, nz, U=0.05)
+    ranks = [mrlbm.Solver("D3Q19", nx, ny, nz, 0.7, "projective", {}, rank=r, nranks=2, transport="p2p")
+             for r in range(2)]
+    try:
+        with pytest.raises(mrlbm.MRLBMError, match="INVALID_ARGUMENT"):
+            ranks[0].set_moments(distributed.slab_of(m0, 2, 0))
+        with pytest.raises(mrlbm.MRLBMError, match="INVALID_ARGUMENT"):
+            ranks[1].step(1)
+    finally:
+        for s in ranks:
+            s.close()
+
+
 @pytest.mark.parametrize("case", [0, 1])
 def test_p2p_two_processes_ipc_bitwise(case):
     from p2p_worker import run_rank

@@ -9,6 +9,12 @@ as in the library's default segmentation.  Cases: fully periodic, lid-driven
 cavity (walls + moving wall), and open velocity / pressure faces on x and on
 y (regularized, R14) next to walls.
 
+The periodic case carries a uniform mean flow (0.03, -0.02, 0.01): without
+one, the seeded modes decay viscously over 1000 steps on this small box
+(exp(-nu k^2 t) ~ 3e-3 at tau = 0.6), the per-group denominator max|oracle|
+shrinks to ~1e-6 and the metric measures the absolute rounding floor
+(~1e-16) of O(1) populations instead of a relative error (R21).
+
 The oracle runs once per physical case (module cache) and serves the fp64 /
 fp32 x segmentation variants of it."""
 import numpy as np
@@ -47,7 +53,8 @@ def reference(lat, reg, bc):
     if key not in _REF:
         import oracle
         (nx, ny, nz), tau, b = case(bc)
-        m0 = inputs.smooth_state(3, nx, ny, nz, U=0.04)
+        mean = (0.03, -0.02, 0.01) if bc == "periodic" else None
+        m0 = inputs.smooth_state(3, nx, ny, nz, U=0.04, mean_u=mean)
         o = oracle.Oracle(lat, nx, ny, nz, tau, reg, b, threads=THREADS)
         o.set_moments(m0)
         o.step(STEPS)

@@ -1,7 +1,9 @@
 """Host-side checks that need no GPU: the C-ABI library loads and exports
 every symbol include/mrlbm.h declares, argument validation, slab partition,
 and the product path fails loudly (no CPU fallback) without a device."""
+import os
 import re
+import sys
 from pathlib import Path
 
 import numpy as np
@@ -157,3 +159,40 @@ def test_slab_neighbours_and_p2p_guards():
     assert distributed.slab_axis_periodic({}, 3) and distributed.slab_axis_periodic({"x-": {"kind": "wall"}}, 2)
     assert not distributed.slab_axis_periodic({"z-": {"kind": "wall"}}, 3)
     assert mrlbm.TRANSPORTS == {"nccl": 0, "p2p": 1} and mrlbm.P2P_HANDLE_BYTES == 512
+
+
+def test_bench_refuses_mismatched_world_size():
+    """bench.py never prints a line whose rank count differs from --gpus."""
+    import subprocess
+    import sys
+    env = dict(os.environ, WORLD_SIZE="2", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, str(ROOT / "bench.py"), "--gpus", "1"], capture_output=True, text=True,
+                       env=env, timeout=120)
+    assert r.returncode == 2 and r.stdout.strip() == "", (r.returncode, r.stdout, r.stderr)
+
+
+def test_bench_configs_weak_and_strong():
+    sys.path.insert(0, str(ROOT))
+    import bench
+    c = bench.build_config("C5", "fp64", 8)
+    assert (c.nx, c.ny, c.nz) == (1024, 1024, 1024) and c.nodes // 8 == 1024 * 1024 * 128
+    c = bench.build_config("C5", "fp64", 1)
+    assert (c.nx, c.ny, c.nz) == (1024, 1024, 128)
+    c = bench.build_config("C5", "fp64", 4, strong=True)
+    assert c.nz == 1024
+    c = bench.build_config("C4", "fp32", 2, strong=True)
+    assert (c.nx, c.ny, c.nz, c.precision) == (512, 512, 512, "fp32")
+    c = bench.build_config("C2", "fp64", 1)
+    assert (c.nx, c.ny, c.regularization) == (4096, 4096, "recursive")
+
+
+def test_input_slabs_are_slices_of_the_global_field():
+    """a rank's slab generated alone equals its slice of the global initial state"""
+    from paper_conf_sc_valero_laravgr23_b200 import configs, inputs
+    g = inputs.perturbed_rest(3, 21, 13, 17)
+    for lo, hi in ((0, 5), (5, 11), (11, 17)):
+        assert np.array_equal(inputs.perturbed_rest(3, 21, 13, 17, lo=lo, hi=hi, chunk=3), g[:, lo:hi])
+    g2 = inputs.perturbed_rest(2, 19, 23)
+    assert np.array_equal(inputs.perturbed_rest(2, 19, 23, lo=7, hi=16), g2[:, 7:16])
+    c = configs.c5(nx=16, ny=12, nz=24)
+    assert np.array_equal(c.initial_moments(lo=6, hi=12), c.initial_moments()[:, 6:12])
