@@ -18,6 +18,7 @@ using mr::StepArgs;
 
 struct Variant {
     int TA, TB, S, BW;
+    int CL;            // CTAs per cluster along B (3D; 1 = no clusters)
     size_t smem;
     void (*step)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t);
     void (*step_push)(const CUtensorMap &, const StepArgs &, dim3, cudaStream_t); // P2P boundary layers (or null)
@@ -32,26 +33,54 @@ struct Variant {
 
 inline int grid_for(long long n) { return (int)std::min<long long>((n + 255) / 256, 148LL * 16); }
 
-template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB, bool WITH_PUSH = false> Variant make_variant()
+// one launch of a step-kernel instance: grid (tiles A, tiles B, segments);
+// CL > 1 launches clusters of CL CTAs along grid.y (cudaLaunchKernelEx)
+template <class KF> inline void launch_step(KF kernel, int CL, int threads, size_t smem, const CUtensorMap &map,
+                                            const StepArgs &a, dim3 grid, cudaStream_t st)
+{
+    if (CL <= 1) {
+        kernel<<<grid, threads, smem, st>>>(map, a);
+        return;
+    }
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = dim3(threads, 1, 1);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 1;
+    attr[0].val.clusterDim.y = CL;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaLaunchKernelEx(&cfg, kernel, map, a);
+}
+
+template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB, bool WITH_PUSH = false, int CL = 1>
+Variant make_variant()
 {
     using L = mr::Lattice<LAT>;
-    using SM = mr::StepSmem<LAT, Real, TA, TB, S>;
+    using SM = mr::StepSmem<LAT, Real, TA, TB, S, CL>;
     Variant v;
     v.TA = TA;
     v.TB = TB;
     v.S = S;
     v.BW = SM::BW;
+    v.CL = CL;
     v.smem = SM::bytes;
-    v.kernel_fn = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB>;
+    v.kernel_fn = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, false, CL>;
     v.step = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
-        mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB><<<grid, TA * TB, SM::bytes, st>>>(map, a);
+        launch_step(mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, false, CL>, CL, TA * TB, SM::bytes, map, a,
+                    grid, st);
     };
     v.step_push = nullptr;
     v.kernel_fn_push = nullptr;
     if constexpr (WITH_PUSH) {
-        v.kernel_fn_push = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true>;
+        v.kernel_fn_push = (const void *)mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true, CL>;
         v.step_push = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
-            mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true><<<grid, TA * TB, SM::bytes, st>>>(map, a);
+            launch_step(mr::mrlbm_step_kernel<LAT, REC, Real, TA, TB, S, MINB, true, CL>, CL, TA * TB, SM::bytes, map,
+                        a, grid, st);
         };
     }
     v.set = [](const double *in, void *buf, mr::GridArgs g, cudaStream_t st) {
@@ -118,9 +147,9 @@ template <int LAT, int COLL, typename Real> StVariant make_st()
 
 
 // per-lattice tables (one translation unit each)
-Variant pick_d2q9(bool rec, bool f32, int tile);
-Variant pick_d3q19(bool rec, bool f32, int tile);
-Variant pick_d3q27(bool rec, bool f32, int tile);
+Variant pick_d2q9(bool rec, bool f32, int tile, int cluster);
+Variant pick_d3q19(bool rec, bool f32, int tile, int cluster);
+Variant pick_d3q27(bool rec, bool f32, int tile, int cluster);
 StVariant select_st(int lat, int coll, int prec);
 // moments (eqs 1-3) of dense fp64 populations [Q][N] -> dense fp64 [M][N] (set_populations)
 void moments_of_populations(int lat, double *pops, double *mom, int nx, int rows, cudaStream_t st);

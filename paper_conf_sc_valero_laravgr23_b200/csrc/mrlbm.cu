@@ -56,13 +56,13 @@ using mrd::StVariant;
 using mrd::select_st;
 using mrd::grid_for;
 
-Variant select_variant(int lat, int reg, int prec, int tile)
+Variant select_variant(int lat, int reg, int prec, int tile, int cluster)
 {
     const bool R = reg == MRLBM_RECURSIVE;
     const bool F = prec == MRLBM_FP32;
-    if (lat == MRLBM_D2Q9) return mrd::pick_d2q9(R, F, tile);
-    if (lat == MRLBM_D3Q19) return mrd::pick_d3q19(R, F, tile);
-    return mrd::pick_d3q27(R, F, tile);
+    if (lat == MRLBM_D2Q9) return mrd::pick_d2q9(R, F, tile, cluster);
+    if (lat == MRLBM_D3Q19) return mrd::pick_d3q19(R, F, tile, cluster);
+    return mrd::pick_d3q27(R, F, tile, cluster);
 }
 
 int env_int(const char *name, int dflt)
@@ -180,7 +180,7 @@ void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st, bool p
         a.c2_end = ce2;
         nseg += (ce2 - cb2 + a.seg_len - 1) / a.seg_len;
     }
-    dim3 grid(h->tilesA * h->tilesB, nseg);
+    dim3 grid(h->tilesA, h->tilesB, nseg);
     if (push) h->var.step_push(h->tmap[src], a, grid, st);
     else h->var.step(h->tmap[src], a, grid, st);
     h->kernels++;
@@ -592,7 +592,7 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
         f.u_profile = nullptr;
     }
 
-    h->var = select_variant(lattice, reg, o.precision, env_int("MRLBM_TILE", 0));
+    h->var = select_variant(lattice, reg, o.precision, env_int("MRLBM_TILE", 0), env_int("MRLBM_CLUSTER", 0));
     for (const void *fn : {h->var.kernel_fn, h->var.kernel_fn_push}) {
         if (!fn) continue;
         if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)h->var.smem) != cudaSuccess ||
@@ -660,9 +660,10 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
         if (a.lo_nb) a.kind[4] = mr::BC_PERIODIC; // interior cut: neighbour data in the ghost plane
         if (a.hi_nb) a.kind[5] = mr::BC_PERIODIC;
     }
-    const int TA = h->var.TA, TB = h->var.TB;
+    const int TA = h->var.TA, TB = h->var.TB, CL = h->var.CL;
     h->tilesA = (h->nA + TA - 3) / (TA - 2);
-    h->tilesB = h->D == 3 ? (h->nB + TB - 3) / (TB - 2) : 1;
+    // 3D: CTAs along B; a cluster of CL CTAs owns CL * TB - 2 rows
+    h->tilesB = h->D == 3 ? (h->nB + CL * TB - 3) / (CL * TB - 2) * CL : 1;
     a.tilesA = h->tilesA;
     // Segments along C.  The grid is tiles x segments; pick the segment count
     // that best fills whole waves of resident CTAs (no tail wave), preferring

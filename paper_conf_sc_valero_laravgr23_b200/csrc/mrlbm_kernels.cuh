@@ -99,6 +99,34 @@ __device__ __forceinline__ void tma_load_4d(void *dst, const CUtensorMap *map, u
         "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
         : "memory");
 }
+// thread-block clusters (3D kernels with CL > 1): rank in the cluster, the
+// cluster-wide barrier (release / acquire: shared-memory stores into a peer
+// CTA before the arrive are visible to its threads after the wait), and the
+// shared::cluster address of the same smem location in CTA `rank`
+__device__ __forceinline__ uint32_t cluster_ctarank()
+{
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all()
+{
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t mapa_shared(uint32_t addr, uint32_t rank)
+{
+    uint32_t r;
+    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+    return r;
+}
+__device__ __forceinline__ void st_cluster(uint32_t addr, double v)
+{
+    asm volatile("st.shared::cluster.f64 [%0], %1;" ::"r"(addr), "d"(v) : "memory");
+}
+__device__ __forceinline__ void st_cluster(uint32_t addr, float v)
+{
+    asm volatile("st.shared::cluster.f32 [%0], %1;" ::"r"(addr), "f"(v) : "memory");
+}
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map)
 {
     asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
@@ -117,7 +145,25 @@ __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map)
 // The full tensor bases (D2Q9 / D3Q27 recursive) use the sum-factorised
 // reconstruction, which applies the per-axis Hermite scale and the D1Q3
 // weights itself; their coefficients carry only tscale(h) = 6^-(#axes with h = 0).
-template <int LAT, bool REC> constexpr bool tensor_recon() { return REC && LAT != LAT_D3Q19; }
+// Reconstruction scheme per variant (and the coefficient scale collide_coeffs
+// applies for it):
+//   PAIR      D2Q9 projective: even/odd pairing of i and opp(i); coefficients
+//             times hscale(h) = prod_a 1/(h_a! c_s^{2 h_a})  (eq 11)
+//   TENSOR_W  D2Q9-R, D3Q27-P/R: sum-factorised 1D Hermite synthesis per axis
+//             with the D1Q3 weights folded in (their weights are D1Q3
+//             products); coefficients times tscale(h) = 6^-(#axes with h = 0)
+//   TENSOR_U  D3Q19-P/R: the same synthesis without weights (D3Q19 weights are
+//             not products), coefficients times hscale(h) / 36, then
+//             f_i = (36 w_i) V(c_i) with 36 w_i in {12, 2, 1}
+// Components absent from a basis (projective: n > 2; D3Q19-R: R10) are
+// compile-time zeros in the synthesis, and populations a lattice does not
+// have are never read, so their arithmetic is removed at compile time.
+enum { RECON_PAIR = 0, RECON_TENSOR_W = 1, RECON_TENSOR_U = 2 };
+template <int LAT, bool REC> constexpr int recon_kind()
+{
+    return LAT == LAT_D2Q9 ? (REC ? RECON_TENSOR_W : RECON_PAIR) : (LAT == LAT_D3Q27 ? RECON_TENSOR_W : RECON_TENSOR_U);
+}
+template <int LAT, bool REC> constexpr bool tensor_recon() { return recon_kind<LAT, REC>() == RECON_TENSOR_W; }
 constexpr double tscale(int D, int h0, int h1, int h2)
 {
     const int z = (h0 == 0) + (h1 == 0) + (D == 3 && h2 == 0);
@@ -168,25 +214,27 @@ __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M],
         else return up[0][m0] * up[1][m1] * up[2][m2];
     };
     using I0 = std::integral_constant<int, 0>;
+    constexpr int RK = recon_kind<LAT, REC>();
+    const Real omc_rho = omc * rho;
     static_for<0, B::NH>([&](auto hk) {
         constexpr int k = decltype(hk)::value;
         constexpr int h0 = B::h[k][0], h1 = B::h[k][1], h2 = B::h[k][2];
         constexpr int n = h0 + h1 + h2;
-        constexpr bool TS = tensor_recon<LAT, REC>();
-        constexpr Real sc = Real(hscale(h0, h1, h2));
-        // tensor bases: the weight scale rides on rho and omega (one product per
-        // distinct scale, shared by every component that has it)
-        constexpr Real ts = Real(TS ? tscale(D, h0, h1, h2) : 1.0);
+        // the coefficient's scale (see recon_kind); it rides on rho, omega and
+        // omc * rho, one product per distinct scale shared by every component
+        // that has it (omega * sc is loop-invariant)
+        constexpr Real sc = Real(RK == RECON_TENSOR_W ? tscale(D, h0, h1, h2)
+                                                      : (RK == RECON_TENSOR_U ? hscale(h0, h1, h2) / 36.0
+                                                                              : hscale(h0, h1, h2)));
         constexpr int i0 = (h0 > 0) ? 0 : ((h1 > 0) ? 1 : 2);
         Real val;
         if constexpr (n == 0) {
-            val = TS ? drho * ts : drho;
+            val = sc == Real(1) ? drho : drho * sc;
         } else if constexpr (n == 1) {
-            val = (TS ? rho * ts : rho) * u[i0];
+            val = (rho * sc) * u[i0];
         } else if constexpr (n == 2) {
             constexpr int i1 = (h0 == 2) ? 0 : ((h0 == 1) ? ((h1 > 0) ? 1 : 2) : ((h1 == 2) ? 1 : 2));
-            if constexpr (TS) val = fma(omega * ts, m[pslot<D>(i0, i1)], (omc * rho * ts) * (u[i0] * u[i1]));
-            else val = omega * m[pslot<D>(i0, i1)] + omc * rho * u[i0] * u[i1];
+            val = fma(omega * sc, m[pslot<D>(i0, i1)], (omc_rho * sc) * (u[i0] * u[i1]));
         } else {
             using H0 = std::integral_constant<int, h0>;
             using H1 = std::integral_constant<int, h1>;
@@ -206,11 +254,9 @@ __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M],
             if constexpr (h1 * h2 > 0)
                 aneq = fma(Real(h1 * h2) * Pn[1][2],
                            mono(H0{}, std::integral_constant<int, h1 - 1>{}, std::integral_constant<int, h2 - 1>{}), aneq);
-            if constexpr (TS) val = fma(omega * ts, aneq, (rho * ts) * mono(H0{}, H1{}, H2{}));
-            else val = fma(omega, aneq, rho * mono(H0{}, H1{}, H2{}));
+            val = fma(omega * sc, aneq, (rho * sc) * mono(H0{}, H1{}, H2{}));
         }
-        if constexpr (TS) A[k] = val; // Hermite scale and weights folded into synth3w
-        else A[k] = val * sc;
+        A[k] = val;
     });
 }
 
@@ -274,6 +320,97 @@ __device__ __forceinline__ void reconstruct_tensor(const Real (&A)[Basis<LAT, tr
     });
 }
 
+// ---- 3D sum-factorised synthesis with compile-time absent components.
+// One 1D synthesis maps coefficients (x0, x1, x2) of orders 0, 1, 2 along an
+// axis to values at c = -1, 0, +1:
+//   weighted (TENSOR_W):   g0 = 4 x0 - x2,  g+- = x0 + x2/2 +- x1/2
+//   unweighted (TENSOR_U): g0 = x0 - x2,    g+- = x0 + 2 x2 +- x1
+// An input that is absent (a compile-time zero) is skipped; an output is
+// present if any input it depends on is.
+constexpr bool syn_present(int c, bool p0, bool p1, bool p2) { return c == 0 ? (p0 || p2) : (p0 || p1 || p2); }
+
+template <bool W, bool P0, bool P1, bool P2, typename Real>
+__device__ __forceinline__ void synth_p(Real x0, Real x1, Real x2, Real &gm, Real &g0, Real &gp)
+{
+    Real S;
+    if constexpr (W) {
+        if constexpr (P0 && P2) { S = fma(Real(0.5), x2, x0); g0 = fma(Real(4), x0, -x2); }
+        else if constexpr (P0) { S = x0; g0 = Real(4) * x0; }
+        else if constexpr (P2) { S = Real(0.5) * x2; g0 = -x2; }
+        if constexpr (P1 && (P0 || P2)) { gp = fma(Real(0.5), x1, S); gm = fma(Real(-0.5), x1, S); }
+        else if constexpr (P1) { gp = Real(0.5) * x1; gm = Real(-0.5) * x1; }
+        else if constexpr (P0 || P2) { gp = S; gm = S; }
+        else { gp = gm = Real(0); } // absent (never read)
+        if constexpr (!(P0 || P2)) g0 = Real(0);
+    } else {
+        if constexpr (P0 && P2) { S = fma(Real(2), x2, x0); g0 = x0 - x2; }
+        else if constexpr (P0) { S = x0; g0 = x0; }
+        else if constexpr (P2) { S = x2 + x2; g0 = -x2; }
+        if constexpr (P1 && (P0 || P2)) { gp = S + x1; gm = S - x1; }
+        else if constexpr (P1) { gp = x1; gm = -x1; }
+        else if constexpr (P0 || P2) { gp = S; gm = S; }
+        else { gp = gm = Real(0); } // absent (never read)
+        if constexpr (!(P0 || P2)) g0 = Real(0);
+    }
+}
+
+// presence of T[a][b][cz] (after the z synthesis) and U[a][cy][cz] (after y)
+template <int LAT, bool REC> constexpr bool presT(int a, int b, int cz)
+{
+    return syn_present(cz, hindex<LAT, REC>(a, b, 0) >= 0, hindex<LAT, REC>(a, b, 1) >= 0, hindex<LAT, REC>(a, b, 2) >= 0);
+}
+template <int LAT, bool REC> constexpr bool presU(int a, int cy, int cz)
+{
+    return syn_present(cy, presT<LAT, REC>(a, 0, cz), presT<LAT, REC>(a, 1, cz), presT<LAT, REC>(a, 2, cz));
+}
+
+template <int LAT, bool REC, typename Real>
+__device__ __forceinline__ void reconstruct_tensor3(const Real (&A)[Basis<LAT, REC>::NH], Real (&f)[Lattice<LAT>::Q])
+{
+    using L = Lattice<LAT>;
+    constexpr bool W = recon_kind<LAT, REC>() == RECON_TENSOR_W;
+    auto coef = [&](auto kc) -> Real {
+        constexpr int k = decltype(kc)::value;
+        if constexpr (k < 0) return Real(0);
+        else return A[k];
+    };
+    Real T[3][3][3]; // [h_x][h_y][c_z + 1]
+    static_for<0, 9>([&](auto abk) {
+        constexpr int a = decltype(abk)::value / 3, b = decltype(abk)::value % 3;
+        constexpr int k0 = hindex<LAT, REC>(a, b, 0), k1 = hindex<LAT, REC>(a, b, 1), k2 = hindex<LAT, REC>(a, b, 2);
+        synth_p<W, (k0 >= 0), (k1 >= 0), (k2 >= 0)>(coef(std::integral_constant<int, k0>{}),
+                                                     coef(std::integral_constant<int, k1>{}),
+                                                     coef(std::integral_constant<int, k2>{}), T[a][b][0], T[a][b][1],
+                                                     T[a][b][2]);
+    });
+    Real U[3][3][3]; // [h_x][c_y + 1][c_z + 1]
+    static_for<0, 9>([&](auto azk) {
+        constexpr int a = decltype(azk)::value / 3, zi = decltype(azk)::value % 3;
+        synth_p<W, presT<LAT, REC>(a, 0, zi - 1), presT<LAT, REC>(a, 1, zi - 1), presT<LAT, REC>(a, 2, zi - 1)>(T[a][0][zi], T[a][1][zi], T[a][2][zi],
+                                                                      U[a][0][zi], U[a][1][zi], U[a][2][zi]);
+    });
+    Real V[3][3][3]; // [c_x + 1][c_y + 1][c_z + 1]
+    static_for<0, 9>([&](auto yzk) {
+        constexpr int yi = decltype(yzk)::value / 3, zi = decltype(yzk)::value % 3;
+        synth_p<W, presU<LAT, REC>(0, yi - 1, zi - 1), presU<LAT, REC>(1, yi - 1, zi - 1),
+                presU<LAT, REC>(2, yi - 1, zi - 1)>(
+            U[0][yi][zi], U[1][yi][zi], U[2][yi][zi], V[0][yi][zi], V[1][yi][zi], V[2][yi][zi]);
+    });
+    static_for<0, L::Q>([&](auto ik) {
+        constexpr int i = decltype(ik)::value;
+        constexpr int xi = L::c[i][0] + 1, yi = L::c[i][1] + 1, zi = L::c[i][2] + 1;
+        if constexpr (W) {
+            f[i] = V[xi][yi][zi];
+        } else {
+            constexpr int m36 = int(L::w[i] * 36.0 + 0.5); // 12, 2 or 1 (D3Q19)
+            static_assert(m36 == 12 || m36 == 2 || m36 == 1, "TENSOR_U weights");
+            if constexpr (m36 == 1) f[i] = V[xi][yi][zi];
+            else if constexpr (m36 == 2) f[i] = V[xi][yi][zi] + V[xi][yi][zi];
+            else f[i] = Real(12) * V[xi][yi][zi];
+        }
+    });
+}
+
 // Multiply-accumulate by a small compile-time integer.
 template <int K, typename Real> __device__ __forceinline__ void acc_int(Real &s, Real v)
 {
@@ -290,7 +427,10 @@ __device__ __forceinline__ void reconstruct(const Real (&A)[Basis<LAT, REC>::NH]
 {
     using L = Lattice<LAT>;
     using B = Basis<LAT, REC>;
-    if constexpr (tensor_recon<LAT, REC>()) {
+    if constexpr (recon_kind<LAT, REC>() != RECON_PAIR && Lattice<LAT>::D == 3) {
+        reconstruct_tensor3<LAT, REC, Real>(A, f);
+        return;
+    } else if constexpr (tensor_recon<LAT, REC>()) {
         reconstruct_tensor<LAT, Real>(A, f);
         return;
     }
@@ -461,7 +601,9 @@ __device__ __forceinline__ float rcp_nr(float x)
 // thread's slot in the exchange plane (stride NT), holding the movers that
 // went through shared memory (SHFL: only those with c_b != 0); the others are
 // read from fown; wt weights arrivals on an open face (R14).
-template <int LAT, typename Real, int NT, bool SHFL>
+// NT: exchange-plane slot stride; UPOFF: extra offset of the c_b = +1 movers'
+// own position (cluster layout: their slot rows start at row -1)
+template <int LAT, typename Real, int NT, bool SHFL, int UPOFF = 0>
 __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *fl, const Real (&fown)[Lattice<LAT>::Q],
                                                               int bbA, int bbB, int bbC, Real rho_own,
                                                               const StepArgs *p, int nx_in, int ny_in, bool open)
@@ -479,7 +621,7 @@ __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *f
         const bool xC = (cm != 0) && (cm == bbC);
         if (xA || xB || xC) {
             Real v;
-            if constexpr (SHFL && X::bmover(k)) v = fl[X::bslot(k) * NT];
+            if constexpr (SHFL && X::bmover(k)) v = fl[X::bslot(k) * NT + (cb > 0 ? UPOFF : 0)];
             else if constexpr (!SHFL && X::moving(k)) v = fl[X::slot(k) * NT];
             else v = fown[k];
             constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
@@ -593,9 +735,20 @@ template <class L, bool SHFL> constexpr int xslot_of(int k)
     return Axes<L>::moving(k) ? Axes<L>::slot(k) : -1;
 }
 
-template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
+// exchange-plane row of window row r for mover k (cluster layout: the slots of
+// the c_b = +1 movers start at row -1, those of the c_b = -1 movers end at row TB)
+template <class L, int CL, int k> __device__ __forceinline__ int xrow(int r)
+{
+    return r + ((CL > 1 && Axes<L>::cb(k) > 0) ? 1 : 0);
+}
+
+template <int LAT, typename Real, int TA, int TB, int S, int CL = 1> struct StepSmem {
     using L = Lattice<LAT>;
     static constexpr int NT = TA * TB;
+    // cluster of CL CTAs stacked along B (3D): each exchange-plane slot has one
+    // extra row -- row -1 for the c_b = +1 movers, row TB for the c_b = -1
+    // movers -- that the neighbouring CTA of the cluster fills through DSMEM
+    static constexpr int RS = (CL > 1) ? (TB + 1) * TA : NT; // elements per slot
     // 3D tiles one warp wide: populations moving only along A are exchanged
     // with warp shuffles, only the c_b != 0 movers go through shared memory
     static constexpr bool SHFL = L::D == 3 && TA == 32;
@@ -606,24 +759,30 @@ template <int LAT, typename Real, int TA, int TB, int S> struct StepSmem {
     static constexpr int BW = (TA + AL - 1 + AL - 1) / AL * AL;
     static constexpr size_t box_elems = size_t(L::M) * TB * BW;
     static constexpr size_t stage_elems = (box_elems * sizeof(Real) + 127) / 128 * 128 / sizeof(Real);
-    static constexpr size_t F_elems = size_t(NX) * NT; // one exchange plane
+    static constexpr size_t F_elems = size_t(NX) * RS; // one exchange plane
     // two exchange planes (alternating layers) -> one __syncthreads per layer
     static constexpr size_t bytes = (S * stage_elems + 2 * F_elems) * sizeof(Real) + S * sizeof(uint64_t) + 128;
 };
 
 // PUSH: the P2P-transport instance for a rank's boundary layers (peer stores);
 // the plain instance carries none of that code
-template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB, bool PUSH = false>
+// CL > 1 (3D): launched in clusters of CL CTAs along B (grid.y); the CTAs of a
+// cluster stack their windows and only the cluster's outermost rows are halo
+// rows (owned rows per cluster CL*TB - 2 instead of CL*(TB - 2)); movers that
+// cross an inner CTA boundary are stored straight into the neighbour CTA's
+// exchange plane (DSMEM) and the per-layer barrier is cluster-wide.
+template <int LAT, bool REC, typename Real, int TA, int TB, int S, int MINB, bool PUSH = false, int CL = 1>
 __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_constant__ CUtensorMap tmap,
                                                             const StepArgs p)
 {
     using L = Lattice<LAT>;
     using X = Axes<L>;
     constexpr int D = L::D, Q = L::Q, M = L::M;
-    constexpr int HB = (D == 3) ? 1 : 0; // halo rows along B
     constexpr int NT = TA * TB;
-    using SM = StepSmem<LAT, Real, TA, TB, S>;
+    using SM = StepSmem<LAT, Real, TA, TB, S, CL>;
     constexpr bool SHFL = SM::SHFL;
+    static_assert(CL == 1 || (D == 3 && SHFL), "clusters: 3D one-warp-wide tiles only");
+    constexpr int RS = SM::RS;
 
     extern __shared__ __align__(128) unsigned char smem_raw[];
     Real *stage = reinterpret_cast<Real *>(smem_raw);
@@ -632,14 +791,20 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
 
     const int tid = threadIdx.x;
     const int tx = tid % TA, ty = tid / TA;
-    const int tA = blockIdx.x % p.tilesA, tB = blockIdx.x / p.tilesA;
+    // grid: x = tile along A, y = tile along B (CL consecutive CTAs = one
+    // cluster), z = sweep segment
+    const int tA = blockIdx.x;
+    const int kcl = (CL > 1) ? int(cluster_ctarank()) : 0;
     const int a0 = tA * (TA - 2) - 1;
-    const int b0 = (D == 3) ? tB * (TB - 2) - 1 : 0;
+    const int b0 = (D == 3) ? (int(blockIdx.y) / CL) * (CL * TB - 2) - 1 + kcl * TB : 0;
     const int a = a0 + tx, b = b0 + ty;
     const int nA = p.nA, nB = p.nB, nC = p.nC;
+    // window rows owned by this CTA: all but the cluster's outermost rows
+    const int row_lo = (D == 3 && kcl == 0) ? 1 : 0;
+    const int row_hi = (D == 3 && kcl == CL - 1) ? TB - 2 : TB - 1;
 
-    const bool second = (int)blockIdx.y >= p.nseg1;
-    const int c0 = second ? p.c2_begin + ((int)blockIdx.y - p.nseg1) * p.seg_len : p.c_begin + blockIdx.y * p.seg_len;
+    const bool second = (int)blockIdx.z >= p.nseg1;
+    const int c0 = second ? p.c2_begin + ((int)blockIdx.z - p.nseg1) * p.seg_len : p.c_begin + blockIdx.z * p.seg_len;
     const int c1 = min(c0 + p.seg_len, second ? p.c2_end : p.c_end);
     if (c0 >= c1) return;
     const int boxA = ((a0 + p.padA) / SM::AL) * SM::AL; // aligned TMA box origin (a0 + padA >= 0)
@@ -664,17 +829,17 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     // periodic ghost column / row (a = -1, nA; b = -1, nB), whose storage the
     // owning edge nodes refresh at every store (see store_ghosts)
     const bool valid = FAST || ((inA || (perA && (a == -1 || a == nA))) && (inB || (perB && (b == -1 || b == nB))));
-    const bool interior = tx >= 1 && tx < TA - 1 && ty >= HB && ty < TB - HB;
+    const bool interior = tx >= 1 && tx < TA - 1 && ty >= row_lo && ty <= row_hi;
     const bool owner = FAST ? interior : (interior && inA && inB);
     // SHFL: every lane of an interior row runs the streaming code (a warp is one
     // row, so the shuffles see all 32 lanes); only owners store
-    const bool stream_lane = SHFL ? (ty >= HB && ty < TB - HB) : owner;
+    const bool stream_lane = SHFL ? (ty >= row_lo && ty <= row_hi) : owner;
     // open faces in this CTA's window (CTA-uniform, so that the weighted and the
     // plain streaming bodies never diverge inside a warp)
-    const int tilesB_ = gridDim.x / p.tilesA;
-    const bool cta_open = !FAST && ((p.kind[0] >= BC_VELOCITY && tA == 0) || (p.kind[1] >= BC_VELOCITY && tA == p.tilesA - 1) ||
-                                    (D == 3 && ((p.kind[2] >= BC_VELOCITY && tB == 0) ||
-                                                (p.kind[3] >= BC_VELOCITY && tB == tilesB_ - 1))));
+    // (a superset: the weighted body is also correct where no node is open)
+    const bool cta_open = !FAST && ((p.kind[0] >= BC_VELOCITY && a0 < 0) || (p.kind[1] >= BC_VELOCITY && a0 + TA - 1 >= nA - 1) ||
+                                    (D == 3 && ((p.kind[2] >= BC_VELOCITY && b0 <= 0) ||
+                                                (p.kind[3] >= BC_VELOCITY && b0 + TB - 1 >= nB - 1))));
     // ghost shift of an owner on a periodic edge: a = 0 -> column nA, a = nA-1 -> column -1
     const int gA = (FAST || !perA) ? 0 : (a == 0 ? nA : (a == nA - 1 ? -nA : 0));
     const int gB = (D == 2 || !perB) ? 0 : (b == 0 ? nB : (b == nB - 1 ? -nB : 0));
@@ -704,7 +869,10 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         for (int s = 0; s < S; s++) mbar_init(&full[s], 1);
         fence_barrier_init();
     }
-    __syncthreads();
+    // clusters: every CTA of the cluster is running (its shared memory may
+    // receive DSMEM stores) once this barrier completes
+    if constexpr (CL > 1) cluster_sync_all();
+    else __syncthreads();
     constexpr uint32_t stage_bytes = uint32_t(SM::box_elems * sizeof(Real)); // bytes one TMA box delivers
     if (tid == 0) {
         for (int s = 0; s < S && s < nl; s++) {
@@ -804,19 +972,41 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
             collide_coeffs<LAT, REC, Real>(m, omega, A);
             rho_own = Real(1) + m[0];
             reconstruct<LAT, REC, Real>(A, fown);
-            static_for<0, Q>([&](auto kk) {
-                constexpr int xs = xslot_of<L, SM::SHFL>(decltype(kk)::value);
-                if constexpr (xs >= 0) Fl[xs * NT + tid] = fown[decltype(kk)::value];
-            });
         } else {
-#pragma unroll
-            for (int q = 0; q < SM::NX; q++) Fl[q * NT + tid] = Real(0);
 #pragma unroll
             for (int q = 0; q < Q; q++) fown[q] = Real(0);
         }
-        // one barrier per layer: the other exchange plane was last read before
-        // this barrier, and every thread has read stage s
-        __syncthreads();
+        static_for<0, Q>([&](auto kk) {
+            constexpr int k = decltype(kk)::value;
+            constexpr int xs = xslot_of<L, SM::SHFL>(k);
+            if constexpr (xs >= 0) Fl[xs * RS + xrow<L, CL, k>(ty) * TA + tx] = fown[k];
+        });
+        if constexpr (CL > 1) {
+            // movers leaving through an inner cluster boundary go straight into
+            // the neighbour CTA's exchange plane: row 0's c_b = -1 movers become
+            // row TB of CTA kcl - 1, row TB-1's c_b = +1 movers row -1 of kcl + 1
+            if (ty == 0 && kcl > 0) {
+                const uint32_t base = mapa_shared(smem_u32(Fl), uint32_t(kcl - 1));
+                static_for<0, Q>([&](auto kk) {
+                    constexpr int k = decltype(kk)::value;
+                    if constexpr (X::cb(k) < 0)
+                        st_cluster(base + uint32_t((X::bslot(k) * RS + TB * TA + tx) * sizeof(Real)), fown[k]);
+                });
+            }
+            if (ty == TB - 1 && kcl < CL - 1) {
+                const uint32_t base = mapa_shared(smem_u32(Fl), uint32_t(kcl + 1));
+                static_for<0, Q>([&](auto kk) {
+                    constexpr int k = decltype(kk)::value;
+                    if constexpr (X::cb(k) > 0)
+                        st_cluster(base + uint32_t((X::bslot(k) * RS + tx) * sizeof(Real)), fown[k]);
+                });
+            }
+        }
+        // one barrier per layer (cluster-wide with CL > 1): the other exchange
+        // plane was last read before this barrier, and every thread has read
+        // stage s
+        if constexpr (CL > 1) cluster_sync_all();
+        else __syncthreads();
         if (tid == 0 && it + S < nl) {
             mbar_expect_tx(&full[s], stage_bytes);
             tma_load_4d(stage + s * SM::stage_elems, &tmap, &full[s], boxA, b0 + p.padB, 0, plane_of(c + S));
@@ -844,7 +1034,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                         } else {
                             Real v;
                             constexpr int xs = xslot_of<L, SM::SHFL>(k);
-                            if constexpr (xs >= 0) v = Fl[xs * NT + (ty - cb) * TA + (tx - ca)];
+                            if constexpr (xs >= 0) v = Fl[xs * RS + xrow<L, CL, k>(ty - cb) * TA + (tx - ca)];
                             else if constexpr (ca != 0) v = __shfl_sync(0xffffffffu, fown[k], tx - ca);
                             else v = fown[k];
                             if constexpr (OPEN) {
@@ -863,7 +1053,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
                 pull(std::integral_constant<int, 1>{}); // assigns Z (= X in the two-set scheme)
                 // halfway bounce-back at walls (R12, R13), out of line
                 if (bbA | bbB | bbC) {
-                    const RVec<Real, M> d = bounce_back<LAT, Real, NT, SM::SHFL>(Fl + tid, fown, bbA, bbB, bbC, rho_own, &p,
+                    const RVec<Real, M> d = bounce_back<LAT, Real, RS, SM::SHFL, (CL > 1 ? TA : 0)>(Fl + tid, fown, bbA, bbB, bbC, rho_own, &p,
                                                                              nx_in, ny_in, OPEN);
 #pragma unroll
                     for (int q = 0; q < M; q++) Y[q] += d.v[q];

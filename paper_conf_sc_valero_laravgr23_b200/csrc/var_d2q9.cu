@@ -3,10 +3,10 @@
 
 namespace mrd {
 
-Variant pick_d2q9(bool rec, bool f32, int tile)
+Variant pick_d2q9(bool rec, bool f32, int tile, int cluster)
 {
-    if (rec) return f32 ? pick<mr::LAT_D2Q9, true, float>(tile) : pick<mr::LAT_D2Q9, true, double>(tile);
-    return f32 ? pick<mr::LAT_D2Q9, false, float>(tile) : pick<mr::LAT_D2Q9, false, double>(tile);
+    if (rec) return f32 ? pick<mr::LAT_D2Q9, true, float>(tile, cluster) : pick<mr::LAT_D2Q9, true, double>(tile, cluster);
+    return f32 ? pick<mr::LAT_D2Q9, false, float>(tile, cluster) : pick<mr::LAT_D2Q9, false, double>(tile, cluster);
 }
 
 } // namespace mrd

@@ -3,10 +3,10 @@
 
 namespace mrd {
 
-Variant pick_d3q27(bool rec, bool f32, int tile)
+Variant pick_d3q27(bool rec, bool f32, int tile, int cluster)
 {
-    if (rec) return f32 ? pick<mr::LAT_D3Q27, true, float>(tile) : pick<mr::LAT_D3Q27, true, double>(tile);
-    return f32 ? pick<mr::LAT_D3Q27, false, float>(tile) : pick<mr::LAT_D3Q27, false, double>(tile);
+    if (rec) return f32 ? pick<mr::LAT_D3Q27, true, float>(tile, cluster) : pick<mr::LAT_D3Q27, true, double>(tile, cluster);
+    return f32 ? pick<mr::LAT_D3Q27, false, float>(tile, cluster) : pick<mr::LAT_D3Q27, false, double>(tile, cluster);
 }
 
 } // namespace mrd

@@ -5,13 +5,17 @@
 
 namespace mrd {
 
+// 3D default: clusters of two CTAs along B (see mrlbm_step_kernel, CL)
+constexpr bool kClusterDefault = false;
+
 // Tile shapes: 2D one row of 128 threads (126 interior
 // nodes); 3D either 32 x 8 threads (30 x 6 interior, 2 CTAs/SM) or 32 x 16
 // threads (30 x 14 interior, 1 CTA/SM).  tile = 0: library default, 1: 32x8,
 // 2: 32x16 (MRLBM_TILE overrides, for tuning).
-template <int LAT, bool REC, typename Real> Variant pick(int tile)
+template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
 {
     if constexpr (LAT == mr::LAT_D2Q9) {
+        (void)cluster;
         // deeper TMA rings trade resident CTAs for bytes in flight (tuning: MRLBM_TILE)
         if (tile == 1) return make_variant<LAT, REC, Real, 128, 1, 4, 4>();
         if (tile == 2) return make_variant<LAT, REC, Real, 128, 1, 6, 4>();
@@ -21,13 +25,21 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile)
         constexpr bool f64 = sizeof(Real) == 8;
         // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
         constexpr bool small_only = LAT == mr::LAT_D3Q27 && f64;
+        const bool dflt = tile == 0;
         if (tile == 0) tile = (LAT == mr::LAT_D3Q19 || small_only) ? 1 : 2;
         // TMA ring depth: with the A-movers exchanged by shuffles the fp64 32x8
         // tile fits three stages at two CTAs per SM; the 32x16 tile (one CTA
         // per SM) takes four in fp32
         // the library defaults also carry the P2P push instance
         constexpr bool small_default = LAT == mr::LAT_D3Q19 || small_only;
-        if (tile == 1 || small_only) return make_variant<LAT, REC, Real, 32, 8, 3, 2, small_default>();
+        // clusters of 2 CTAs along B (DSMEM mover exchange, no halo rows between
+        // them): cluster = 0 library default, 1 off, 2 on (MRLBM_CLUSTER)
+        const bool cl2 = dflt && (cluster == 2 || (cluster == 0 && kClusterDefault));
+        if (tile == 1 || small_only) {
+            if (cl2) return make_variant<LAT, REC, Real, 32, 8, 3, 2, small_default, 2>();
+            return make_variant<LAT, REC, Real, 32, 8, 3, 2, small_default>();
+        }
+        if (cl2) return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 4), 1, !small_default, 2>();
         return make_variant<LAT, REC, Real, 32, 16, (f64 ? 2 : 4), 1, !small_default>();
     }
 }
