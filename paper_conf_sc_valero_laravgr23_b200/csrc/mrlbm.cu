@@ -855,8 +855,12 @@ mrlbm_status mrlbm_step(mrlbm_t h, int64_t n)
 {
     if (!h || n < 0) return fail(MRLBM_ERR_INVALID_ARGUMENT, "bad step count");
     if (h->group_mode) return fail(MRLBM_ERR_INVALID_ARGUMENT, "slab-group handle: use mrlbm_step_group");
-    // Batches of kGraphSteps single-rank steps are replayed from a captured graph.
-    while (h->nranks == 1 && n >= kGraphSteps) {
+    // Batches of kGraphSteps single-rank or P2P-transport steps are replayed
+    // from a captured graph (the P2P wait / signal kernels read and write the
+    // device counters at run time, so a replay orders itself).  NCCL steps stay
+    // eager: their launch overhead is < 1% of a C5w step, and NCCL capture
+    // cannot be validated on the one-GPU test box.
+    while ((h->nranks == 1 || h->p2p) && n >= kGraphSteps) {
         const int par = h->cur;
         if (!h->graph[par]) {
             cudaGraph_t g;

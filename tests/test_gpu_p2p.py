@@ -64,6 +64,38 @@ def test_p2p_in_process_bitwise(case, P):
     assert np.array_equal(got, ref), f"max diff {np.abs(got - ref).max()}"
 
 
+@pytest.mark.parametrize("case", [0, 3])
+def test_p2p_in_process_graph_replay_bitwise(case):
+    """P2P steps in batches (captured and replayed as CUDA graphs of 32 steps,
+    each rank on its own stream, ordered only by the device counters)."""
+    from paper_conf_sc_valero_laravgr23_b200 import mrlbm
+    lat, reg, (nx, ny, nz), b, precision = CASES[case]
+    D = 2 if lat == "D2Q9" else 3
+    P, steps = 2, 70
+    with mrlbm.Solver(lat, nx, ny, nz, 0.7, reg, b, precision=precision) as one:
+        one.set_moments(inputs.smooth_state(D, nx, ny, nz, U=0.05))
+        one.step(steps)
+        ref = one.get_moments()
+    ranks = [mrlbm.Solver(lat, nx, ny, nz, 0.7, reg, b, precision=precision, rank=r, nranks=P, transport="p2p")
+             for r in range(P)]
+    try:
+        handles = [s.p2p_handle() for s in ranks]
+        for s in ranks:
+            distributed.p2p_connect(s, handles, distributed.slab_axis_periodic(b, D))
+        m0 = inputs.smooth_state(D, nx, ny, nz, U=0.05)
+        for r, s in enumerate(ranks):
+            s.set_moments(distributed.slab_of(m0, P, r))
+        for s in ranks:
+            s.step(steps)   # 2 graph replays of 32 steps + 6 eager steps, enqueued rank after rank
+        for s in ranks:
+            s.sync()
+        got = np.concatenate([s.get_moments() for s in ranks], axis=1)
+    finally:
+        for s in ranks:
+            s.close()
+    assert np.array_equal(got, ref), f"max diff {np.abs(got - ref).max()}"
+
+
 def test_p2p_set_before_connect_is_refused():
     """The neighbours' ghost planes can only be filled once connected: setting
     the state of a P2P handle before mrlbm_p2p_connect is an error, not a
