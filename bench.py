@@ -426,6 +426,9 @@ def run_gpu(args, rank, world, local_rank):
 
     # end to end through the public C-ABI with host buffers: upload (pinned),
     # K steps, download -- all inside the timed region
+    if args.no_e2e:  # side runs whose host state would not fit twice in pinned memory
+        return finish_line(args, s, c, st, world, rank, local_rank, dist, name, nodes_local, rep_ms, ms_step, ms,
+                           launches, blk_steps, blk_ms, blk_mlups, clocks, value, comm, None)
     import torch as _t
     pinned_in = _t.from_numpy(m_local).pin_memory()
     pinned_out = _t.empty_like(pinned_in).pin_memory()
@@ -445,6 +448,12 @@ def run_gpu(args, rank, world, local_rank):
            "h2d_bytes_per_step": roofline.M_OF[c.lattice] * 8 * c.nodes / args.steps,
            "d2h_bytes_per_step": roofline.M_OF[c.lattice] * 8 * c.nodes / args.steps,
            "job": "mrlbm_set_moments (pinned host) + mrlbm_step(K) + mrlbm_get_moments (pinned host), wall clock"}
+    return finish_line(args, s, c, st, world, rank, local_rank, dist, name, nodes_local, rep_ms, ms_step, ms,
+                       launches, blk_steps, blk_ms, blk_mlups, clocks, value, comm, e2e)
+
+
+def finish_line(args, s, c, st, world, rank, local_rank, dist, name, nodes_local, rep_ms, ms_step, ms, launches,
+                blk_steps, blk_ms, blk_mlups, clocks, value, comm, e2e):
     finite_ok = True
     try:
         s.check_finite()
@@ -476,14 +485,18 @@ def run_gpu(args, rank, world, local_rank):
             "config": dict(workload_config(c, world, args.strong), method=args.method,
                            **({"transport": args.transport} if world > 1 else {})),
             "per_gpu_mlups": value / world,
-            "reps": {"n": reps, "steps_each": args.steps, "ms_per_step": [t / args.steps for t in rep_ms],
+            "reps": {"n": len(rep_ms), "steps_each": args.steps, "ms_per_step": [t / args.steps for t in rep_ms],
                      "median_ms_per_step": ms_step,
                      "spread_pct": 100.0 * (max(rep_ms) - min(rep_ms)) / ms},
             "sustained": {"blocks": 5, "steps_per_block": blk_steps, "block_ms": blk_ms,
                           "mlups": blk_mlups, "median_mlups": statistics.median(blk_mlups)},
-            "roofline": rl, "clocks": clocks, "e2e": e2e, "gpu_launches": launches,
+            "roofline": rl, "clocks": clocks, "gpu_launches": launches,
             "kernel": s.kernel_config(), "finite": finite_ok,
             "gpus_active": world, "comm": comm}
+    if e2e is not None:
+        line["e2e"] = e2e
+    else:
+        line["e2e_skipped"] = "--no-e2e (side run: the host state does not fit twice in pinned memory)"
     s.close()
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(c, seconds=args.cpu_seconds)
@@ -517,6 +530,7 @@ def main():
                     help="N > 1 halo transport: NCCL send/recv (default) or peer-memory pushes fused into the step")
     ap.add_argument("--cpu-seconds", type=float, default=16.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true", help="skip the host-buffer e2e leg (side runs only)")
     ap.add_argument("--ref-side", type=int, default=1024, help="reference arm: max sample sub-domain side")
     ap.add_argument("--ref-seconds", type=float, default=60.0, help="reference arm: target timed seconds")
     args = ap.parse_args()

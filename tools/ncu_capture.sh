@@ -6,7 +6,7 @@ mkdir -p gpurun_out
 for cfg in "$@"; do set -- $cfg
   R=gpurun_out/prof_${TAG}_$1_$2
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:mrlbm_step -s 5 -c 1 \
-    -o /tmp/prof_${TAG}_$1_$2 -f python bench.py --config $1 --precision $2 --steps 10 --warmup 3 --no-cpu-baseline \
+    -o /tmp/prof_${TAG}_$1_$2 -f python bench.py --config $1 --precision $2 --steps 10 --warmup 3 --no-cpu-baseline --no-e2e \
     > ${R}.log 2>&1; tail -1 ${R}.log
   ncu -i /tmp/prof_${TAG}_$1_$2.ncu-rep --page raw --csv > ${R}_raw.csv 2>/dev/null
   ncu -i /tmp/prof_${TAG}_$1_$2.ncu-rep --page source --csv --print-source sass > ${R}_sass.csv 2>/dev/null

@@ -1,6 +1,6 @@
-"""Per-step cost of the slab decomposition on ONE GPU: the
-C5w workload (D3Q19-R channel 1024 x 1024 x 128, fp64) as 1 rank vs P = 2 ranks
-in one process, with the P2P transport (pushes fused into the boundary
+"""Per-step cost of the slab decomposition on ONE GPU: a
+D3Q19-R channel (fp64) of 1024 x 1024 x (128 P) as 1 rank vs P = 2 ranks of one
+C5w slab (1024 x 1024 x 128) each, in one process, with the P2P transport (pushes fused into the boundary
 launches, device counters, graph-replayed) and with the slab-group transport
 (device-to-device ghost copies).  All ranks share the one GPU, so the total
 work is equal and the difference is the decomposition's overhead: extra
@@ -34,17 +34,17 @@ def timed(fn, syncs, reps=5):
     return out[len(out) // 2]
 
 
-def main(steps=128):
-    c = configs.c5(nz=128)
+def main(steps=128, P=2):
+    c = configs.c5(nz=128 * P)
     m0 = c.initial_moments()
     args = (c.lattice, c.nx, c.ny, c.nz, c.tau, c.regularization, c.boundary)
-    res = {"workload": "C5w: D3Q19 recursive channel 1024x1024x128 fp64", "steps": steps}
+    res = {"workload": f"D3Q19 recursive channel 1024x1024x{128 * P} fp64: 1 rank vs {P} ranks of 1024x1024x128",
+           "steps": steps}
     with mrlbm.Solver(*args) as one:
         one.set_moments(m0)
         one.step(64)
         res["one_rank_ms_per_step"] = timed(lambda: one.step(steps), [one]) / steps * 1e3
-    # P2P, 2 ranks in one process (own streams), batches replayed as graphs
-    P = 2
+    # P2P, P ranks in one process (own streams), batches replayed as graphs
     ranks = [mrlbm.Solver(*args, rank=r, nranks=P, transport="p2p") for r in range(P)]
     hs = [s.p2p_handle() for s in ranks]
     for s in ranks:
@@ -59,7 +59,7 @@ def main(steps=128):
     res["p2p_2ranks_ms_per_step"] = timed(run_p2p, ranks) / steps * 1e3
     for s in ranks:
         s.close()
-    # slab group (D2D copies), 2 ranks
+    # slab group (D2D copies), P ranks
     grp = [mrlbm.Solver(*args, rank=r, nranks=P) for r in range(P)]
     for r, s in enumerate(grp):
         s.set_moments(distributed.slab_of(m0, P, r))
