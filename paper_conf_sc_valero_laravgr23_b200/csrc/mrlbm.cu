@@ -781,14 +781,44 @@ mrlbm_status mrlbm_get_moments_device(mrlbm_t h, double *dst_dev, int64_t count)
     return p2p_check(h);
 }
 
+// Host I/O of the moment representation goes through a bounded device staging
+// buffer, a chunk of whole layers at a time (a 2D copy gathers the chunk's
+// M strided pieces of the [M][nC][nB][nA] host array): a state that fills the
+// GPU (C5 1024^3 fp64 in two copies) needs no full-size fp64 staging copy.
+static const size_t kStageBytes = size_t(1) << 30;
+
+static int64_t stage_layers(const mrlbm_ctx *h)
+{
+    const size_t per_layer = (size_t)h->M * h->nA * h->nB * sizeof(double);
+    return std::max<int64_t>(1, std::min<int64_t>(h->nC, (int64_t)(kStageBytes / per_layer)));
+}
+
 mrlbm_status mrlbm_set_moments(mrlbm_t h, const double *src, int64_t count)
 {
     if (!h || !src) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
     if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
-    mrlbm_status s = ensure_io(h, (size_t)count * sizeof(double));
+    if (h->repr == MRLBM_DISTRIBUTIONS) { // ST: one full-size staging copy
+        mrlbm_status s = ensure_io(h, (size_t)count * sizeof(double));
+        if (s) return s;
+        MR_CUDA(cudaMemcpyAsync(h->io, src, (size_t)count * sizeof(double), cudaMemcpyHostToDevice, h->stream));
+        return mrlbm_set_moments_device(h, h->io, count);
+    }
+    if (h->p2p && !h->p2p_connected)
+        return fail(MRLBM_ERR_INVALID_ARGUMENT, "P2P transport: mrlbm_p2p_connect before setting the state");
+    const int64_t plane = (int64_t)h->nA * h->nB, N = local_nodes(h), L = stage_layers(h);
+    mrlbm_status s = ensure_io(h, (size_t)h->M * L * plane * sizeof(double));
     if (s) return s;
-    MR_CUDA(cudaMemcpyAsync(h->io, src, (size_t)count * sizeof(double), cudaMemcpyHostToDevice, h->stream));
-    s = mrlbm_set_moments_device(h, h->io, count);
+    for (int64_t c0 = 0; c0 < h->nC; c0 += L) {
+        const int64_t len = std::min<int64_t>(L, h->nC - c0);
+        MR_CUDA(cudaMemcpy2DAsync(h->io, (size_t)(len * plane) * sizeof(double), src + c0 * plane,
+                                  (size_t)N * sizeof(double), (size_t)(len * plane) * sizeof(double), (size_t)h->M,
+                                  cudaMemcpyHostToDevice, h->stream));
+        mr::GridArgs g = grid_args(h);
+        g.nC = (int)len;
+        h->var.set(h->io, (char *)node0(h, h->cur) + (size_t)c0 * h->pstride * h->wbytes, g, h->stream);
+        MR_CUDA(cudaGetLastError());
+    }
+    s = p2p_prologue(h);
     if (s) return s;
     MR_CUDA(cudaStreamSynchronize(h->stream));
     return MRLBM_OK;
@@ -798,13 +828,30 @@ mrlbm_status mrlbm_get_moments(mrlbm_t h, double *dst, int64_t count)
 {
     if (!h || !dst) return fail(MRLBM_ERR_INVALID_ARGUMENT, "null argument");
     if (count != (int64_t)h->M * local_nodes(h)) return fail(MRLBM_ERR_BUFFER_SIZE, "count != M * N_local");
-    mrlbm_status s = ensure_io(h, (size_t)count * sizeof(double));
+    if (h->repr == MRLBM_DISTRIBUTIONS) {
+        mrlbm_status s = ensure_io(h, (size_t)count * sizeof(double));
+        if (s) return s;
+        s = mrlbm_get_moments_device(h, h->io, count);
+        if (s) return s;
+        MR_CUDA(cudaMemcpyAsync(dst, h->io, (size_t)count * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+        MR_CUDA(cudaStreamSynchronize(h->stream));
+        return MRLBM_OK;
+    }
+    const int64_t plane = (int64_t)h->nA * h->nB, N = local_nodes(h), L = stage_layers(h);
+    mrlbm_status s = ensure_io(h, (size_t)h->M * L * plane * sizeof(double));
     if (s) return s;
-    s = mrlbm_get_moments_device(h, h->io, count);
-    if (s) return s;
-    MR_CUDA(cudaMemcpyAsync(dst, h->io, (size_t)count * sizeof(double), cudaMemcpyDeviceToHost, h->stream));
+    for (int64_t c0 = 0; c0 < h->nC; c0 += L) {
+        const int64_t len = std::min<int64_t>(L, h->nC - c0);
+        mr::GridArgs g = grid_args(h);
+        g.nC = (int)len;
+        h->var.get((const char *)node0(h, h->cur) + (size_t)c0 * h->pstride * h->wbytes, h->io, g, h->stream);
+        MR_CUDA(cudaGetLastError());
+        MR_CUDA(cudaMemcpy2DAsync(dst + c0 * plane, (size_t)N * sizeof(double), h->io,
+                                  (size_t)(len * plane) * sizeof(double), (size_t)(len * plane) * sizeof(double),
+                                  (size_t)h->M, cudaMemcpyDeviceToHost, h->stream));
+    }
     MR_CUDA(cudaStreamSynchronize(h->stream));
-    return MRLBM_OK;
+    return p2p_check(h);
 }
 
 mrlbm_status mrlbm_get_populations(mrlbm_t h, double *dst, int64_t count)

@@ -76,19 +76,36 @@ def main():
     md = [f"# ncu --set full summaries ({tag})\n",
           "One launch of the fused step kernel per workload (`ncu --set full --clock-control none "
           "--import-source on -k regex:mrlbm_step -s 5 -c 1`), cold-cache and serialised by ncu.\n",
-          "| workload | kernel | time | DRAM bytes/launch | DRAM GB/s | DRAM % peak | regs | block x grid | "
-          "warps active % | issue % | fp64 pipe % | fma pipe % | L2 hit % |",
-          "|---|---|---|---|---|---|---|---|---|---|---|---|---|"]
+          "| workload | kernel | time | DRAM bytes/launch | traffic / algorithmic (2 M w per LUP) | DRAM GB/s | "
+          "regs | block x grid | warps active % | issue % | fp64 pipe % | fma pipe % | L2 hit % | warp-inst / LUP | "
+          "ALU ceiling (MLUPS, unit) |",
+          "|---|---|---|---|---|---|---|---|---|---|---|---|---|---|---|"]
     for key, rep in zip(args[0::2], args[1::2]):
         r = read_rep(rep)
         r["tag"] = tag
         r["report"] = Path(rep).name
         summ[key] = r
+        # LUPs per launch and algorithmic bytes from the key: C?-LAT-REG-PREC-NXxNYxNZ
+        parts = key.split("-")
+        lat, prec = parts[1], parts[3]
+        nx, ny, nz = (int(v) for v in parts[4].split("x"))
+        lups = nx * ny * nz
+        M = 6 if lat == "D2Q9" else 10
+        alg = 2 * M * (8 if prec == "fp64" else 4) * lups
+        r["lups_per_launch"] = lups
+        r["algorithmic_bytes_per_launch"] = alg
+        dur = r.get("duration", 0) or 1e-30
+        ceil = {u: lups / (dur * r[k] / 100.0) / 1e6 for u, k in
+                (("issue", "issue_active_pct"), ("fp64", "fp64_pipe_pct"), ("fma", "fma_pipe_pct")) if r.get(k)}
+        cu = min(ceil, key=ceil.get) if ceil else None
         md.append(f"| {key} | `{r['kernel'][:60]}` | {r.get('duration', 0) * 1e6:.1f} us | "
-                  f"{r.get('dram_bytes_per_launch', 0) / 1e9:.3f} GB | {r.get('dram_gbs', 0):.0f} | "
-                  f"{r.get('dram_pct_peak', 0):.1f} | {r.get('registers', 0):.0f} | {r.get('block', 0):.0f} x "
+                  f"{r.get('dram_bytes_per_launch', 0) / 1e9:.3f} GB | "
+                  f"{r.get('dram_bytes_per_launch', 0) / alg:.3f} | {r.get('dram_gbs', 0):.0f} | "
+                  f"{r.get('registers', 0):.0f} | {r.get('block', 0):.0f} x "
                   f"{r.get('grid', 0):.0f} | {r.get('warps_active_pct', 0):.1f} | {r.get('issue_active_pct', 0):.1f} | "
-                  f"{r.get('fp64_pipe_pct', 0):.1f} | {r.get('fma_pipe_pct', 0):.1f} | {r.get('l2_hit_pct', 0):.1f} |")
+                  f"{r.get('fp64_pipe_pct', 0):.1f} | {r.get('fma_pipe_pct', 0):.1f} | {r.get('l2_hit_pct', 0):.1f} | "
+                  f"{r.get('warp_inst', 0) / lups:.2f} | "
+                  f"{(f'{ceil[cu]:.0f} ({cu})') if cu else '-'} |")
     summ_path.write_text(json.dumps(summ, indent=1, sort_keys=True))
     (ROOT / "profiles" / f"ncu_{tag}.md").write_text("\n".join(md) + "\n")
     print("\n".join(md))
