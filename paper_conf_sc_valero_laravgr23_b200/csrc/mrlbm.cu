@@ -678,9 +678,13 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
         const long long slots = (long long)std::max(occ, 1) * nsm;
         long long seg = env_int("MRLBM_SEG", 0);
         if (seg <= 0 && h->D == 2) {
-            // 2D: short segments keep the resident CTAs on nearby rows, so the
-            // halo columns they share are L2 hits (measured: 24 rows best on C2)
-            seg = 24;
+            // 2D: short segments keep the resident CTAs on a narrow band of
+            // rows (halo rows shared by consecutive segments are L2 hits, the
+            // DRAM streams stay local); each segment recomputes two halo rows.
+            // Measured on C2 (profiles/segsweep_r02.jsonl, seg2d_r02.jsonl):
+            // fp64 (HBM-bound) 0.84 at 24 rows -> 0.883 at 10-14; fp32
+            // (issue-bound, pays the halo rows) best at 16-18.
+            seg = h->prec == MRLBM_FP64 ? 12 : 16;
         } else if (seg <= 0) {
             // 3D: segment lengths 32..96; best wave fill, ties to the longer
             double best = -1.0;
