@@ -20,6 +20,9 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         if (tile == 1) return make_variant<LAT, REC, Real, 128, 1, 4, 4>();
         if (tile == 2) return make_variant<LAT, REC, Real, 128, 1, 6, 4>();
         if (tile == 3) return make_variant<LAT, REC, Real, 128, 1, 8, 3>();
+        // fp32: a stage is only 3 KB, so deep rings fit at 5 CTAs per SM
+        if (tile == 4) return make_variant<LAT, REC, Real, 128, 1, 8, 5>();
+        if (tile == 5) return make_variant<LAT, REC, Real, 128, 1, 12, 5>();
         return make_variant<LAT, REC, Real, 128, 1, 4, 5, true>();
     } else {
         constexpr bool f64 = sizeof(Real) == 8;
