@@ -23,7 +23,13 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         // fp32: a stage is only 3 KB, so deep rings fit at 5 CTAs per SM
         if (tile == 4) return make_variant<LAT, REC, Real, 128, 1, 8, 5>();
         if (tile == 5) return make_variant<LAT, REC, Real, 128, 1, 12, 5>();
-        return make_variant<LAT, REC, Real, 128, 1, 4, 5, true>();
+        if (tile == 6) return make_variant<LAT, REC, Real, 128, 1, 5, 4>();
+        if (tile == 7) return make_variant<LAT, REC, Real, 128, 1, 6, 6>();
+        if (tile == 8) return make_variant<LAT, REC, Real, 128, 1, 4, 5>(); // round-1 default
+        // default: a 6-deep TMA ring; fp64 at 4 CTAs/SM (6 x 6.2 KB stages), fp32 at 6
+        // (measured C2: fp64 0.90 -> 0.916, fp32 0.80 -> 0.82; profiles/ring2d_b_r02.jsonl)
+        if constexpr (sizeof(Real) == 8) return make_variant<LAT, REC, Real, 128, 1, 6, 4, true>();
+        else return make_variant<LAT, REC, Real, 128, 1, 6, 6, true>();
     } else {
         constexpr bool f64 = sizeof(Real) == 8;
         // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
@@ -38,6 +44,9 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         // clusters of 2 CTAs along B (DSMEM mover exchange, no halo rows between
         // them): cluster = 0 library default, 1 off, 2 on (MRLBM_CLUSTER)
         const bool cl2 = dflt && (cluster == 2 || (cluster == 0 && kClusterDefault));
+        if constexpr (!f64) { // fp32 32x16: deeper TMA ring (tuning: MRLBM_TILE=3)
+            if (tile == 3) return make_variant<LAT, REC, Real, 32, 16, 6, 1>();
+        }
         if (tile == 1 || small_only) {
             if (cl2) return make_variant<LAT, REC, Real, 32, 8, 3, 2, small_default, 2>();
             return make_variant<LAT, REC, Real, 32, 8, 3, 2, small_default>();
