@@ -181,6 +181,7 @@ void launch_range(mrlbm_ctx *h, int src, int cb, int ce, cudaStream_t st, bool p
         nseg += (ce2 - cb2 + a.seg_len - 1) / a.seg_len;
     }
     dim3 grid(h->tilesA, h->tilesB, nseg);
+    if (a.rastG > 0) grid = dim3(h->tilesA * h->tilesB, 1, nseg); // grouped launch order (kernel remaps)
     if (push) h->var.step_push(h->tmap[src], a, grid, st);
     else h->var.step(h->tmap[src], a, grid, st);
     h->kernels++;
@@ -665,6 +666,11 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     // 3D: CTAs along B; a cluster of CL CTAs owns CL * TB - 2 rows
     h->tilesB = h->D == 3 ? (h->nB + CL * TB - 3) / (CL * TB - 2) * CL : 1;
     a.tilesA = h->tilesA;
+    a.tilesB = h->tilesB;
+    // 3D launch order: groups of MRLBM_RAST B-tiles (tuning; default 0 = the plain
+    // (A, B) grid: measured C3 -2% / -5% at groups of 4 / 8, C5 +0.6%, C4 -0.3%,
+    // profiles/ab_r03.md)
+    a.rastG = (h->D == 3 && CL == 1) ? std::max(0, env_int("MRLBM_RAST", 0)) : 0;
     // Segments along C.  The grid is tiles x segments; pick the segment count
     // that best fills whole waves of resident CTAs (no tail wave), preferring
     // longer segments (each segment re-reads one halo layer at each end).

@@ -42,7 +42,9 @@ struct StepArgs {
     int seg_len;            // layers per CTA segment
     int nseg1;              // segments of the first range; grid.y beyond it covers [c2_begin, c2_end)
     int c2_begin, c2_end;   // optional second range (a slab's first and last layer in one launch)
-    int tilesA;             // tiles along A (grid.x = tilesA * tilesB)
+    int tilesA;             // tiles along A
+    int tilesB;             // tiles along B (3D)
+    int rastG;              // 3D, CL = 1: grid.x = tilesA * tilesB in launch groups of rastG B-tiles (0: grid (A, B))
     int lo_nb, hi_nb;       // 1 if layer -1 / nC exists (periodic wrap or ghost plane)
     int wrapC;              // 1: layer c lives in plane wrap(c)+1 (single-rank periodic C)
     int c_offset;           // global index of local layer 0 (profiles)
@@ -260,6 +262,65 @@ __device__ __forceinline__ void collide_coeffs(const Real (&m)[Lattice<LAT>::M],
     });
 }
 
+// Post-collision coefficients of D3Q19 for the U36 synthesis (synth_p U36, SYN_U36) (eq 10; eqs 12-13 through
+// the pair-sum closed form of the recursion, R8), all divided by 36 and with
+// no per-component Hermite scale (the synthesis applies it per axis).  With
+// r = rho/36, P'_ab = Pi^neq_ab / 36 = Pi_ab/36 - r u_a u_b:
+//   order 0: (rho - 1)/36      order 1: r u_a      order 2: Pi*_ab = r u_a u_b + omega P'_ab
+//   order 3 (recursive), e.g. (2,1,0): r ux^2 uy + omega (P'xx uy + 2 P'xy ux)
+//                                      = uy Pi*_xx + ux R_xy,   R_ab = 2 omega P'_ab
+//   order 4, e.g. (2,2,0): r ux^2 uy^2 + omega (P'xx uy^2 + P'yy ux^2 + 4 P'xy ux uy)
+//                          = uy a_210 + ux (omega P'yy ux + R_xy uy)
+// (the same coefficients collide_coeffs forms term by term, regrouped)
+template <bool REC, typename Real>
+__device__ __forceinline__ void collide_u36(const Real (&m)[10], Real omega, Real (&A)[Basis<LAT_D3Q19, REC>::NH])
+{
+    constexpr Real k = Real(1.0 / 36.0);
+    const Real drho = m[0];
+    const Real r = fma(drho, k, k);
+    const Real ux = m[1], uy = m[2], uz = m[3];
+    const Real rx = r * ux, ry = r * uy, rz = r * uz;
+    const Real rxx = rx * ux, ryy = ry * uy, rzz = rz * uz, rxy = rx * uy, rxz = rx * uz, ryz = ry * uz;
+    const Real pxx = fma(m[4], k, -rxx), pyy = fma(m[5], k, -ryy), pzz = fma(m[6], k, -rzz);
+    const Real pxy = fma(m[7], k, -rxy), pxz = fma(m[8], k, -rxz), pyz = fma(m[9], k, -ryz);
+    A[0] = drho * k;
+    A[1] = rx;
+    A[2] = ry;
+    A[3] = rz;
+    if constexpr (REC) {
+        const Real oxx = omega * pxx, oyy = omega * pyy, ozz = omega * pzz;
+        const Real w2 = omega + omega;
+        const Real Rxy = w2 * pxy, Rxz = w2 * pxz, Ryz = w2 * pyz;
+        const Real Sxx = rxx + oxx, Syy = ryy + oyy, Szz = rzz + ozz;
+        A[4] = Sxx;
+        A[5] = Syy;
+        A[6] = Szz;
+        A[7] = fma(Real(0.5), Rxy, rxy);
+        A[8] = fma(Real(0.5), Rxz, rxz);
+        A[9] = fma(Real(0.5), Ryz, ryz);
+        // basis order (lattice.cuh): 210 201 120 021 102 012 220 202 022
+        const Real a210 = fma(uy, Sxx, ux * Rxy), a201 = fma(uz, Sxx, ux * Rxz);
+        const Real a120 = fma(ux, Syy, uy * Rxy), a021 = fma(uz, Syy, uy * Ryz);
+        const Real a102 = fma(ux, Szz, uz * Rxz), a012 = fma(uy, Szz, uz * Ryz);
+        A[10] = a210;
+        A[11] = a201;
+        A[12] = a120;
+        A[13] = a021;
+        A[14] = a102;
+        A[15] = a012;
+        A[16] = fma(ux, fma(oyy, ux, Rxy * uy), uy * a210);
+        A[17] = fma(ux, fma(ozz, ux, Rxz * uz), uz * a201);
+        A[18] = fma(uy, fma(ozz, uy, Ryz * uz), uz * a021);
+    } else {
+        A[4] = fma(omega, pxx, rxx);
+        A[5] = fma(omega, pyy, ryy);
+        A[6] = fma(omega, pzz, rzz);
+        A[7] = fma(omega, pxy, rxy);
+        A[8] = fma(omega, pxz, rxz);
+        A[9] = fma(omega, pyz, ryz);
+    }
+}
+
 template <int LAT, bool REC> constexpr int hindex(int a, int b, int c)
 {
     for (int k = 0; k < Basis<LAT, REC>::NH; k++)
@@ -329,11 +390,22 @@ __device__ __forceinline__ void reconstruct_tensor(const Real (&A)[Basis<LAT, tr
 // present if any input it depends on is.
 constexpr bool syn_present(int c, bool p0, bool p1, bool p2) { return c == 0 ? (p0 || p2) : (p0 || p1 || p2); }
 
-template <bool W, bool P0, bool P1, bool P2, typename Real>
+// U36: unweighted with the per-axis Hermite scale applied here (coefficients
+// from collide_u36): g0 = x0 - 3/2 x2, g+- = x0 + 3 x2 +- 3 x1
+template <bool W, bool P0, bool P1, bool P2, typename Real, bool U36 = false>
 __device__ __forceinline__ void synth_p(Real x0, Real x1, Real x2, Real &gm, Real &g0, Real &gp)
 {
     Real S;
-    if constexpr (W) {
+    if constexpr (U36 && !W) {
+        if constexpr (P0 && P2) { S = fma(Real(3), x2, x0); g0 = fma(Real(-1.5), x2, x0); }
+        else if constexpr (P0) { S = x0; g0 = x0; }
+        else if constexpr (P2) { S = Real(3) * x2; g0 = Real(-1.5) * x2; }
+        if constexpr (P1 && (P0 || P2)) { gp = fma(Real(3), x1, S); gm = fma(Real(-3), x1, S); }
+        else if constexpr (P1) { gp = Real(3) * x1; gm = Real(-3) * x1; }
+        else if constexpr (P0 || P2) { gp = S; gm = S; }
+        else { gp = gm = Real(0); }
+        if constexpr (!(P0 || P2)) g0 = Real(0);
+    } else if constexpr (W) {
         if constexpr (P0 && P2) { S = fma(Real(0.5), x2, x0); g0 = fma(Real(4), x0, -x2); }
         else if constexpr (P0) { S = x0; g0 = Real(4) * x0; }
         else if constexpr (P2) { S = Real(0.5) * x2; g0 = -x2; }
@@ -364,7 +436,7 @@ template <int LAT, bool REC> constexpr bool presU(int a, int cy, int cz)
     return syn_present(cy, presT<LAT, REC>(a, 0, cz), presT<LAT, REC>(a, 1, cz), presT<LAT, REC>(a, 2, cz));
 }
 
-template <int LAT, bool REC, typename Real>
+template <int LAT, bool REC, typename Real, bool U36 = false>
 __device__ __forceinline__ void reconstruct_tensor3(const Real (&A)[Basis<LAT, REC>::NH], Real (&f)[Lattice<LAT>::Q])
 {
     using L = Lattice<LAT>;
@@ -378,7 +450,7 @@ __device__ __forceinline__ void reconstruct_tensor3(const Real (&A)[Basis<LAT, R
     static_for<0, 9>([&](auto abk) {
         constexpr int a = decltype(abk)::value / 3, b = decltype(abk)::value % 3;
         constexpr int k0 = hindex<LAT, REC>(a, b, 0), k1 = hindex<LAT, REC>(a, b, 1), k2 = hindex<LAT, REC>(a, b, 2);
-        synth_p<W, (k0 >= 0), (k1 >= 0), (k2 >= 0)>(coef(std::integral_constant<int, k0>{}),
+        synth_p<W, (k0 >= 0), (k1 >= 0), (k2 >= 0), Real, U36>(coef(std::integral_constant<int, k0>{}),
                                                      coef(std::integral_constant<int, k1>{}),
                                                      coef(std::integral_constant<int, k2>{}), T[a][b][0], T[a][b][1],
                                                      T[a][b][2]);
@@ -386,14 +458,14 @@ __device__ __forceinline__ void reconstruct_tensor3(const Real (&A)[Basis<LAT, R
     Real U[3][3][3]; // [h_x][c_y + 1][c_z + 1]
     static_for<0, 9>([&](auto azk) {
         constexpr int a = decltype(azk)::value / 3, zi = decltype(azk)::value % 3;
-        synth_p<W, presT<LAT, REC>(a, 0, zi - 1), presT<LAT, REC>(a, 1, zi - 1), presT<LAT, REC>(a, 2, zi - 1)>(T[a][0][zi], T[a][1][zi], T[a][2][zi],
+        synth_p<W, presT<LAT, REC>(a, 0, zi - 1), presT<LAT, REC>(a, 1, zi - 1), presT<LAT, REC>(a, 2, zi - 1), Real, U36>(T[a][0][zi], T[a][1][zi], T[a][2][zi],
                                                                       U[a][0][zi], U[a][1][zi], U[a][2][zi]);
     });
     Real V[3][3][3]; // [c_x + 1][c_y + 1][c_z + 1]
     static_for<0, 9>([&](auto yzk) {
         constexpr int yi = decltype(yzk)::value / 3, zi = decltype(yzk)::value % 3;
         synth_p<W, presU<LAT, REC>(0, yi - 1, zi - 1), presU<LAT, REC>(1, yi - 1, zi - 1),
-                presU<LAT, REC>(2, yi - 1, zi - 1)>(
+                presU<LAT, REC>(2, yi - 1, zi - 1), Real, U36>(
             U[0][yi][zi], U[1][yi][zi], U[2][yi][zi], V[0][yi][zi], V[1][yi][zi], V[2][yi][zi]);
     });
     static_for<0, L::Q>([&](auto ik) {
@@ -601,7 +673,7 @@ __device__ __forceinline__ float rcp_nr(float x)
 // thread's slot in the exchange plane (stride NT), holding the movers that
 // went through shared memory (SHFL: only those with c_b != 0); the others are
 // read from fown; wt weights arrivals on an open face (R14).
-// NT: exchange-plane slot stride; UPOFF: extra offset of the c_b = +1 movers'
+// NT: exchange-plane slot stride (0: all of fown is valid); UPOFF: extra offset of the c_b = +1 movers'
 // own position (cluster layout: their slot rows start at row -1)
 template <int LAT, typename Real, int NT, bool SHFL, int UPOFF = 0>
 __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *fl, const Real (&fown)[Lattice<LAT>::Q],
@@ -621,7 +693,8 @@ __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *f
         const bool xC = (cm != 0) && (cm == bbC);
         if (xA || xB || xC) {
             Real v;
-            if constexpr (SHFL && X::bmover(k)) v = fl[X::bslot(k) * NT + (cb > 0 ? UPOFF : 0)];
+            if constexpr (NT == 0) v = fown[k]; // every population passed in registers
+            else if constexpr (SHFL && X::bmover(k)) v = fl[X::bslot(k) * NT + (cb > 0 ? UPOFF : 0)];
             else if constexpr (!SHFL && X::moving(k)) v = fl[X::slot(k) * NT];
             else v = fown[k];
             constexpr int kx = L::c[k][0], ky = L::c[k][1], kz = L::c[k][2];
@@ -793,10 +866,24 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     const int tx = tid % TA, ty = tid / TA;
     // grid: x = tile along A, y = tile along B (CL consecutive CTAs = one
     // cluster), z = sweep segment
-    const int tA = blockIdx.x;
+    // Launch order (3D, no clusters): consecutive CTAs walk groups of rastG
+    // B-neighbours, group by group along A, so that the CTAs sharing a halo row
+    // (B) or halo columns (A) run close together in time and their shared
+    // box rows are L2 hits rather than second DRAM reads.
+    int tA = blockIdx.x, tBi = blockIdx.y;
+    if (D == 3 && CL == 1 && p.rastG > 0) {
+        const int L = blockIdx.x;
+        const int span = p.rastG * p.tilesA;
+        const int grp = L / span;
+        const int w = L - grp * span;
+        const int g0 = grp * p.rastG;
+        const int gsz = min(p.rastG, p.tilesB - g0);
+        tA = w / gsz;
+        tBi = g0 + (w - tA * gsz);
+    }
     const int kcl = (CL > 1) ? int(cluster_ctarank()) : 0;
     const int a0 = tA * (TA - 2) - 1;
-    const int b0 = (D == 3) ? (int(blockIdx.y) / CL) * (CL * TB - 2) - 1 + kcl * TB : 0;
+    const int b0 = (D == 3) ? (tBi / CL) * (CL * TB - 2) - 1 + kcl * TB : 0;
     const int a = a0 + tx, b = b0 + ty;
     const int nA = p.nA, nB = p.nB, nC = p.nC;
     // window rows owned by this CTA: all but the cluster's outermost rows
@@ -825,10 +912,12 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
     // ---- per-thread roles
     const bool perA = p.kind[0] == BC_PERIODIC, perB = p.kind[2] == BC_PERIODIC;
     const bool inA = a >= 0 && a < nA, inB = b >= 0 && b < nB;
-    // a window position holds a real node if it is inside the domain or is the
-    // periodic ghost column / row (a = -1, nA; b = -1, nB), whose storage the
-    // owning edge nodes refresh at every store (see store_ghosts)
-    const bool valid = FAST || ((inA || (perA && (a == -1 || a == nA))) && (inB || (perB && (b == -1 || b == nB))));
+    // Every window position is computed, node or not: positions that hold no
+    // node (pads outside a non-periodic face, TMA out-of-bounds boxes) read
+    // all-zero moments (the buffers are zeroed at creation and only nodes and
+    // periodic ghosts are ever stored), and zero shifted moments (rho - 1 = 0,
+    // u = 0, Pi = 0) collide and reconstruct to exactly zero shifted
+    // populations -- so they publish zeros and the pulls need no predicate.
     const bool interior = tx >= 1 && tx < TA - 1 && ty >= row_lo && ty <= row_hi;
     const bool owner = FAST ? interior : (interior && inA && inB);
     // SHFL: every lane of an interior row runs the streaming code (a warp is one
@@ -955,7 +1044,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         mbar_wait(&full[s], (it / S) & 1);
 
         Real m[M];
-        if (valid) {
+        {
             const Real *st = stage + s * SM::stage_elems + ty * SM::BW + tx + offA;
 #pragma unroll
             for (int q = 0; q < M; q++) m[q] = st[q * (TB * SM::BW)];
@@ -966,15 +1055,17 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         // exist land in accumulators that are never stored)
         Real *Fl = Fs + (it & 1) * SM::F_elems;
         Real fown[Q]; // only the non-moving entries are used after the barrier
-        Real rho_own = Real(1);
-        if (valid) {
+        const Real rho_own = Real(1) + m[0];
+        {
             Real A[Basis<LAT, REC>::NH];
-            collide_coeffs<LAT, REC, Real>(m, omega, A);
-            rho_own = Real(1) + m[0];
-            reconstruct<LAT, REC, Real>(A, fown);
-        } else {
-#pragma unroll
-            for (int q = 0; q < Q; q++) fown[q] = Real(0);
+            if constexpr (LAT == LAT_D3Q19) {
+                // regrouped collision, Hermite scales applied per axis by the synthesis
+                collide_u36<REC, Real>(m, omega, A);
+                reconstruct_tensor3<LAT, REC, Real, true>(A, fown);
+            } else {
+                collide_coeffs<LAT, REC, Real>(m, omega, A);
+                reconstruct<LAT, REC, Real>(A, fown);
+            }
         }
         static_for<0, Q>([&](auto kk) {
             constexpr int k = decltype(kk)::value;

@@ -34,6 +34,26 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         constexpr bool f64 = sizeof(Real) == 8;
         // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
         constexpr bool small_only = LAT == mr::LAT_D3Q27 && f64;
+        // default (tile 0): the paired kernel (step3d.cuh), same tile shapes as
+        // the round-2 defaults; tile 9: the round-2 scalar kernel (A/B)
+        if (tile == 0 && cluster != 2) {
+            if constexpr (LAT == mr::LAT_D3Q19 || small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true>();
+            else return make_variant3<LAT, REC, Real, 16, (f64 ? 2 : 4), 1, true>();
+        }
+        // tile 10: the paired kernel on 32 x 8 tiles at 2 CTAs/SM (A/B for D3Q27 fp32)
+        if (tile == 10) {
+            if constexpr (!small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true>();
+        }
+        // tile 11: the paired kernel with split-phase exchange barriers (A/B)
+        if (tile == 11) {
+            if constexpr (LAT == mr::LAT_D3Q19 || small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true>();
+            else return make_variant3<LAT, REC, Real, 16, (f64 ? 2 : 4), 1, true, true>();
+        }
+        // tile 12: split-phase barriers on 32 x 8 tiles at 2 CTAs/SM (A/B, D3Q27 fp32)
+        if (tile == 12) {
+            if constexpr (!small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true>();
+        }
+        if (tile == 9) tile = 0;
         const bool dflt = tile == 0;
         if (tile == 0) tile = (LAT == mr::LAT_D3Q19 || small_only) ? 1 : 2;
         // TMA ring depth: with the A-movers exchanged by shuffles the fp64 32x8
