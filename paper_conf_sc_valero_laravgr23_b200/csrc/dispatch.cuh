@@ -107,22 +107,24 @@ Variant make_variant()
 }
 
 // the paired 3D kernel (step3d.cuh): same Variant table, TA = 32, no clusters
-template <int LAT, bool REC, typename Real, int TB, int S, int MINB, bool WITH_PUSH = false, bool SPLIT = false> Variant make_variant3()
+template <int LAT, bool REC, typename Real, int TB, int S, int MINB, bool WITH_PUSH = false, bool SPLIT = false,
+          bool ONEBODY = false>
+Variant make_variant3()
 {
     using SM = mr::Step3Smem<LAT, Real, TB, S>;
     Variant v = make_variant<LAT, REC, Real, 32, TB, S, MINB, false, 1>(); // side kernels
     v.BW = SM::BW;
     v.smem = SM::bytes;
-    v.kernel_fn = (const void *)mr::mrlbm_step3_kernel<LAT, REC, Real, TB, S, MINB, false, SPLIT>;
+    v.kernel_fn = (const void *)mr::mrlbm_step3_kernel<LAT, REC, Real, TB, S, MINB, false, SPLIT, ONEBODY>;
     v.step = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
-        mr::mrlbm_step3_kernel<LAT, REC, Real, TB, S, MINB, false, SPLIT><<<grid, 32 * TB, SM::bytes, st>>>(map, a);
+        mr::mrlbm_step3_kernel<LAT, REC, Real, TB, S, MINB, false, SPLIT, ONEBODY><<<grid, 32 * TB, SM::bytes, st>>>(map, a);
     };
     v.step_push = nullptr;
     v.kernel_fn_push = nullptr;
     if constexpr (WITH_PUSH) {
-        v.kernel_fn_push = (const void *)mr::mrlbm_step3_kernel<LAT, REC, Real, TB, S, MINB, true, SPLIT>;
+        v.kernel_fn_push = (const void *)mr::mrlbm_step3_kernel<LAT, REC, Real, TB, S, MINB, true, SPLIT, ONEBODY>;
         v.step_push = [](const CUtensorMap &map, const StepArgs &a, dim3 grid, cudaStream_t st) {
-            mr::mrlbm_step3_kernel<LAT, REC, Real, TB, S, MINB, true, SPLIT><<<grid, 32 * TB, SM::bytes, st>>>(map, a);
+            mr::mrlbm_step3_kernel<LAT, REC, Real, TB, S, MINB, true, SPLIT, ONEBODY><<<grid, 32 * TB, SM::bytes, st>>>(map, a);
         };
     }
     return v;

@@ -510,6 +510,9 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
         mrlbm_destroy(h);
         return s;
     };
+    // the step kernels address a layer's moment planes with 32-bit offsets
+    if (h->pstride >= (1LL << 31))
+        return cleanup_fail(fail(MRLBM_ERR_UNSUPPORTED, "layer too large: M * (nB + 2) * pitch must stay below 2^31 elements"));
 
     if (o.cuda_stream) {
         h->stream = (cudaStream_t)o.cuda_stream;

@@ -1009,14 +1009,15 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
         if (!owner) return;
         Real *o = dst_node + (long long)(c + 1) * p.pstride;
         auto store_plane = [&](Real *o) {
+            const int ms = int(p.mstride); // < 2^31 elements per moment plane (32-bit offsets)
 #pragma unroll
-            for (int q = 0; q < M; q++) o[q * p.mstride] = out[q];
+            for (int q = 0; q < M; q++) o[q * ms] = out[q];
             // periodic ghost copies of edge nodes (also the corner ghosts)
             if (gA | gB) {
                 auto put = [&](int da, int db) {
                     Real *g = o + (long long)db * p.pitch + da;
 #pragma unroll
-                    for (int q = 0; q < M; q++) g[q * p.mstride] = out[q];
+                    for (int q = 0; q < M; q++) g[q * ms] = out[q];
                 };
                 if (gA) put(gA, 0);
                 if (gB) put(0, gB);

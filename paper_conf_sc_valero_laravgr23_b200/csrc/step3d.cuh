@@ -27,6 +27,10 @@ namespace mr {
 // inline every lambda of the step kernel (nvcc otherwise outlines the large
 // ones with a stack frame)
 #define AI __attribute__((always_inline))
+#ifndef MRLBM_Q27_PRODUCT
+#define MRLBM_Q27_PRODUCT 1
+#endif
+constexpr bool Q27_PRODUCT = MRLBM_Q27_PRODUCT;
 
 // ------------------------------------------------------------ pairs over c_m = (-1, +1)
 template <typename Real> struct Pr;
@@ -71,6 +75,15 @@ __device__ __forceinline__ Pr<float> vmul(float c, Pr<float> x) { return {__fmul
 __device__ __forceinline__ Pr<double> vmul(double c, Pr<double> x) { return mkpr(c * x.v.x, c * x.v.y); }
 template <typename Real> __device__ __forceinline__ Real vzero(Real *) { return Real(0); }
 template <typename Real> __device__ __forceinline__ Pr<Real> vzero(Pr<Real> *) { return mkpr(Real(0), Real(0)); }
+// s * x + y with the scalar s broadcast (x, y pairs)
+__device__ __forceinline__ Pr<float> pfma_b(float s, Pr<float> x, Pr<float> y) { return {__ffma2_rn(make_float2(s, s), x.v, y.v)}; }
+__device__ __forceinline__ Pr<double> pfma_b(double s, Pr<double> x, Pr<double> y)
+{
+    return mkpr(fma(s, x.v.x, y.v.x), fma(s, x.v.y, y.v.y));
+}
+// c * x + q with the constant c and the scalar q broadcast
+__device__ __forceinline__ Pr<float> pfma_cb(float c, Pr<float> x, float q) { return {__ffma2_rn(make_float2(c, c), x.v, make_float2(q, q))}; }
+__device__ __forceinline__ Pr<double> pfma_cb(double c, Pr<double> x, double q) { return mkpr(fma(c, x.v.x, q), fma(c, x.v.y, q)); }
 // (S - h x1, S + h x1): one packed FMA with both scalars broadcast
 __device__ __forceinline__ Pr<float> pm_pair(float h, float x1, float S)
 {
@@ -206,6 +219,158 @@ __device__ __forceinline__ void reconstruct_pairs(const Real (&A)[Basis<LAT, REC
     });
 }
 
+// ------------------------------------------------------------ D3Q27 recursive in product form
+// For the full tensor basis the recursive-regularized coefficients are (eqs
+// 10, 12-13; R8)  a*_h = rho u^h + (omega/2) sum_ab Pneq_ab d_a d_b u^h  for
+// every h in {0,1,2}^3 (the pair-sum closed form is this second derivative),
+// and the weighted Hermite synthesis (eq 14) is a tensor product of 1D maps.
+// So every term is separable and the synthesis of each factor is a 1D
+// function of one velocity component:
+//   E(c) = syn(1, u, u^2):  E(0) = 2/3 - u^2,  E(+-1) = 1/6 + u^2/2 +- u/2
+//   D(c) = syn(0, 1, 2u):   D(0) = -2u,        D(+-1) = u +- 1/2
+//   DD(c)= syn(0, 0, 2):    DD(0) = -2,        DD(+-1) = 1
+// (D1Q3 weights w(0) = 2/3, w(1) = 1/6 and the Hermite scales folded in), and
+//   f* = rho ExEyEz + (omega/2)(Pxx DDx Ey Ez + Pyy Ex DDy Ez + Pzz Ex Ey DDz)
+//        + omega (Pxy Dx Dy Ez + Pxz Dx Ey Dz + Pyz Ex Dy Dz).
+// The state is shifted (R16): f~ = f* - Wx Wy Wz with W = E(u = 0); writing
+// E = W + Ehat and rho = 1 + drho, rho ExEyEz - WxWyWz
+//   = [(drho Ex + Ehatx) Ey + Wx Ehaty] Ez + Wx Wy Ehatz   (small terms only).
+// Evaluated x first, then per (cx, cy), then the c_z pair / scalar -- it
+// replaces collide_coeffs + reconstruct_pairs for D3Q27 recursive in fp64
+// (209 instead of 262 FP64 instructions per node) and gives the same
+// populations up to rounding.  Not in fp32: E(+-1) = 1/6 + u^2/2 +- u/2 stored
+// as one fp32 number keeps only ~1.5e-8 of its O(u) part, and the 1000-step
+// parity error grows 3-6x (profiles/r03/probe.txt); keeping the weight and the
+// small part apart costs as many instructions as the sum-factorised form.
+template <typename Real>
+__device__ __forceinline__ void collide_reconstruct_q27r(const Real (&m)[10], Real omega, Real (&f0)[3][3], Pr<Real> (&fp)[3][3])
+{
+    const Real drho = m[0];
+    const Real rho = Real(1) + drho;
+    const Real u[3] = {m[1], m[2], m[3]};
+    // Pi^neq = Pi - rho u u; halves of the diagonal times omega, off-diagonal times omega
+    const Real ru0 = rho * u[0], ru1 = rho * u[1], ru2 = rho * u[2];
+    const Real hw = Real(0.5) * omega;
+    const Real hPxx = hw * fma(-ru0, u[0], m[4]), hPyy = hw * fma(-ru1, u[1], m[5]), hPzz = hw * fma(-ru2, u[2], m[6]);
+    const Real wPxy = omega * fma(-ru0, u[1], m[7]), wPxz = omega * fma(-ru0, u[2], m[8]), wPyz = omega * fma(-ru1, u[2], m[9]);
+    // per-axis 1D factors, index c + 1
+    Real E[3][3], Eh[3][3], Dv[3][3];
+#pragma unroll
+    for (int a = 0; a < 3; a++) {
+        const Real uu = u[a] * u[a];
+        const Real h2 = Real(0.5) * uu;
+        Eh[a][1] = -uu;
+        Eh[a][0] = fma(Real(-0.5), u[a], h2);
+        Eh[a][2] = fma(Real(0.5), u[a], h2);
+        E[a][1] = Real(2.0 / 3.0) - uu;
+        E[a][0] = Real(1.0 / 6.0) + Eh[a][0];
+        E[a][2] = Real(1.0 / 6.0) + Eh[a][2];
+        Dv[a][1] = Real(-2) * u[a];
+        Dv[a][0] = u[a] - Real(0.5);
+        Dv[a][2] = u[a] + Real(0.5);
+    }
+    const Pr<Real> Ez = mkpr(E[2][0], E[2][2]), Dz = mkpr(Dv[2][0], Dv[2][2]), Ehz = mkpr(Eh[2][0], Eh[2][2]);
+    static_for<0, 3>([&](auto xk) {
+        constexpr int xi = decltype(xk)::value;
+        constexpr Real Wx = xi == 1 ? Real(2.0 / 3.0) : Real(1.0 / 6.0);
+        constexpr Real DDx = xi == 1 ? Real(-2) : Real(1);
+        const Real ax = fma(drho, E[0][xi], Eh[0][xi]);  // rho Ex - Wx
+        const Real al = fma(DDx, hPxx, ax);               // + (omega/2) Pxx DDx
+        const Real be = hPyy * E[0][xi];
+        const Real ga = wPxy * Dv[0][xi];
+        const Real ze = hPzz * E[0][xi];
+        const Real de = wPxz * Dv[0][xi];
+        const Real ep = wPyz * E[0][xi];
+        static_for<0, 3>([&](auto yk) {
+            constexpr int yi = decltype(yk)::value;
+            constexpr Real Wy = yi == 1 ? Real(2.0 / 3.0) : Real(1.0 / 6.0);
+            constexpr Real DDy = yi == 1 ? Real(-2) : Real(1);
+            constexpr Real WW = Wx * Wy;
+            const Real Q1 = fma(E[1][yi], al, fma(Wx, Eh[1][yi], fma(DDy, be, ga * Dv[1][yi])));
+            const Real Q2 = ze * E[1][yi];
+            const Real Q3 = fma(de, E[1][yi], ep * Dv[1][yi]);
+            // c_z = 0: Q1 Ez0 - 2 Q2 + Q3 Dz0 + Wx Wy Ehatz0
+            f0[xi][yi] = fma(Q1, E[2][1], fma(Real(-2), Q2, fma(Q3, Dv[2][1], WW * Eh[2][1])));
+            // c_z = -1, +1: Q1 Ez + Q2 + Q3 Dz + Wx Wy Ehatz
+            fp[xi][yi] = pfma_b(Q1, Ez, pfma_b(Q3, Dz, pfma_cb(WW, Ehz, Q2)));
+        });
+    });
+}
+
+// ------------------------------------------------------------ D3Q27 recursive, regrouped
+// The 27 post-collision coefficients of D3Q27 recursive for the weighted
+// synthesis (SYN_W: A_h = tscale(h) a*_h, tscale = 6^-(#axes with h = 0)),
+// with the pair sums of the recursion (eqs 12-13, R8) regrouped so that each
+// order reuses the one below (as collide_u36 for D3Q19).  With
+// S_ab = Pi*_ab = rho u_a u_b + omega P_ab (P = Pi^neq), R_ab = 2 omega P_ab:
+//   a210 = uy S_xx + ux R_xy                      a111 = uz S_xy + (uy R_xz + ux R_yz)/2
+//   a220 = uy a210 + ux (omega P_yy ux + R_xy uy) a211 = uz a210 + ux (R_xz uy + omega P_yz ux)
+//   a221 = uz a220 + ux uy (uy R_xz + ux R_yz)    a222 = uz a221 + ux uy (omega P_zz ux uy + uz (uy R_xz + ux R_yz))
+// and their permutations (each identity is the pair-sum closed form of
+// collide_coeffs, term by term).  ~105 instead of 154 FP32 instructions.
+template <typename Real>
+__device__ __forceinline__ void collide_q27r(const Real (&m)[10], Real omega, Real (&A)[27])
+{
+    constexpr Real t1 = Real(1.0 / 6.0), t2 = Real(1.0 / 36.0), t3 = Real(1.0 / 216.0);
+    const Real drho = m[0];
+    const Real rho = Real(1) + drho;
+    const Real ux = m[1], uy = m[2], uz = m[3];
+    const Real rx = rho * ux, ry = rho * uy, rz = rho * uz;
+    const Real rxx = rx * ux, ryy = ry * uy, rzz = rz * uz, rxy = rx * uy, rxz = rx * uz, ryz = ry * uz;
+    const Real Pxx = m[4] - rxx, Pyy = m[5] - ryy, Pzz = m[6] - rzz;
+    const Real Pxy = m[7] - rxy, Pxz = m[8] - rxz, Pyz = m[9] - ryz;
+    const Real wxx = omega * Pxx, wyy = omega * Pyy, wzz = omega * Pzz;
+    const Real w2 = omega + omega;
+    const Real Rxy = w2 * Pxy, Rxz = w2 * Pxz, Ryz = w2 * Pyz;
+    const Real wxy = omega * Pxy, wxz = omega * Pxz, wyz = omega * Pyz;
+    const Real Sxx = rxx + wxx, Syy = ryy + wyy, Szz = rzz + wzz;
+    const Real Sxy = rxy + wxy, Sxz = rxz + wxz, Syz = ryz + wyz;
+    const Real a210 = fma(uy, Sxx, ux * Rxy), a201 = fma(uz, Sxx, ux * Rxz);
+    const Real a120 = fma(ux, Syy, uy * Rxy), a021 = fma(uz, Syy, uy * Ryz);
+    const Real a102 = fma(ux, Szz, uz * Rxz), a012 = fma(uy, Szz, uz * Ryz);
+    const Real tyz = fma(uy, Rxz, ux * Ryz); // uy R_xz + ux R_yz
+    const Real a111 = fma(uz, Sxy, Real(0.5) * tyz);
+    const Real a220 = fma(ux, fma(wyy, ux, Rxy * uy), uy * a210);
+    const Real a202 = fma(ux, fma(wzz, ux, Rxz * uz), uz * a201);
+    const Real a022 = fma(uy, fma(wzz, uy, Ryz * uz), uz * a021);
+    const Real a211 = fma(uz, a210, ux * fma(Rxz, uy, wyz * ux));
+    const Real a121 = fma(uz, a120, uy * fma(Ryz, ux, wxz * uy));
+    const Real a112 = fma(uy, a102, uz * fma(Ryz, ux, wxy * uz));
+    const Real uxy = ux * uy, uxz = ux * uz, uyz = uy * uz;
+    const Real a221 = fma(uz, a220, uxy * tyz);
+    const Real a212 = fma(uy, a202, uxz * fma(uz, Rxy, ux * Ryz));
+    const Real a122 = fma(ux, a022, uyz * fma(uz, Rxy, uy * Rxz));
+    const Real a222 = fma(uz, a221, uxy * fma(wzz, uxy, uz * tyz));
+    // basis order (lattice.cuh), times tscale
+    A[0] = t3 * drho;
+    A[1] = t2 * rx;
+    A[2] = t2 * ry;
+    A[3] = t2 * rz;
+    A[4] = t2 * Sxx;
+    A[5] = t2 * Syy;
+    A[6] = t2 * Szz;
+    A[7] = t1 * Sxy;
+    A[8] = t1 * Sxz;
+    A[9] = t1 * Syz;
+    A[10] = t1 * a210;
+    A[11] = t1 * a201;
+    A[12] = t1 * a120;
+    A[13] = t1 * a021;
+    A[14] = t1 * a102;
+    A[15] = t1 * a012;
+    A[16] = a111;
+    A[17] = t1 * a220;
+    A[18] = t1 * a202;
+    A[19] = t1 * a022;
+    A[20] = a211;
+    A[21] = a121;
+    A[22] = a112;
+    A[23] = a221;
+    A[24] = a212;
+    A[25] = a122;
+    A[26] = a222;
+}
+
 // ------------------------------------------------------------ exchange-plane slots
 // In-plane movers along B (c_b != 0) go through shared memory: the pairs
 // (c_m = +-1) and the c_m = 0 scalars each get one slot per (c_a, c_b).
@@ -326,7 +491,7 @@ __device__ __forceinline__ void mbar_arrive(uint64_t *bar)
     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 
-template <int LAT, bool REC, typename Real, int TB, int S, int MINB, bool PUSH = false, bool SPLIT = false>
+template <int LAT, bool REC, typename Real, int TB, int S, int MINB, bool PUSH = false, bool SPLIT = false, bool ONEBODY = false>
 __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid_constant__ CUtensorMap tmap,
                                                                    const StepArgs p)
 {
@@ -500,9 +665,18 @@ __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid
         const Real rho_own = Real(1) + m[0];
         {
             Real A[Basis<LAT, REC>::NH];
-            if constexpr (LAT == LAT_D3Q19) collide_u36<REC, Real>(m, omega, A);
-            else collide_coeffs<LAT, REC, Real>(m, omega, A);
-            reconstruct_pairs<LAT, REC, Real>(A, f0, fp);
+            // product form in fp64 only: in fp32 the factors E(c) = w(c) + O(u) round
+            // their small part against the O(1) weight (1000-step parity error
+            // u 7.2e-5 vs 1.9e-5 for the sum-factorised form, profiles/r03/probe.txt)
+            if constexpr (LAT == LAT_D3Q27 && REC && Q27_PRODUCT && sizeof(Real) == 8) {
+                (void)A;
+                collide_reconstruct_q27r<Real>(m, omega, f0, fp);
+            } else {
+                if constexpr (LAT == LAT_D3Q19) collide_u36<REC, Real>(m, omega, A);
+                else if constexpr (LAT == LAT_D3Q27 && REC) collide_q27r<Real>(m, omega, A);
+                else collide_coeffs<LAT, REC, Real>(m, omega, A);
+                reconstruct_pairs<LAT, REC, Real>(A, f0, fp);
+            }
         }
         // publish the c_b != 0 movers
         if constexpr (SPLIT) {
@@ -614,7 +788,9 @@ __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid
     // two accumulator sets with alternating roles (sweep unrolled by two, no
     // accumulator moves) wherever it fits the register file without spills: all
     // but D3Q27 recursive fp64, which keeps three rotating sets
-    if constexpr (!(LAT == LAT_D3Q27 && REC && sizeof(Real) == 8)) {
+    // ONEBODY: one layer body and three rotating sets (half the loop code: the
+    // instruction-cache footprint of the sweep, at 2 M register moves per layer)
+    if constexpr (!ONEBODY && !(LAT == LAT_D3Q27 && REC && sizeof(Real) == 8)) {
         for (int it = 0; it < nl; it += 2) {
             layer(it, accA, accB, accA);
             if (it + 1 < nl) layer(it + 1, accB, accA, accB);

@@ -34,11 +34,20 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         constexpr bool f64 = sizeof(Real) == 8;
         // smem: S TMA stages + two exchange planes; D3Q27 fp64 only fits the small tile
         constexpr bool small_only = LAT == mr::LAT_D3Q27 && f64;
-        // default (tile 0): the paired kernel (step3d.cuh), same tile shapes as
-        // the round-2 defaults; tile 9: the round-2 scalar kernel (A/B)
+        // Defaults (tile 0), from the round-3 one-box A/Bs (profiles/r03/):
+        //  D3Q19 fp64: the scalar kernel (mrlbm_step_kernel, 32 x 8, 2 CTAs/SM) with
+        //         the regrouped collision -- the paired kernel's fp64 pair registers
+        //         cost moves (+8% instructions on C3) and it measured 1-5% slower;
+        //  D3Q19 fp32 and D3Q27: the paired kernel (step3d.cuh) on 32 x 8 tiles at
+        //         2 CTAs/SM (packed FP32; C3 fp32 +3%, C4 fp32 +4% over the scalar
+        //         kernel; C4 fp64 +14% with the product-form D3Q27-R).
+        // tile 9 selects the round-2 default shapes of the scalar kernel (A/B).
         if (tile == 0 && cluster != 2) {
-            if constexpr (LAT == mr::LAT_D3Q19 || small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true>();
-            else return make_variant3<LAT, REC, Real, 16, (f64 ? 2 : 4), 1, true>();
+            if constexpr (LAT == mr::LAT_D3Q27 || !f64) return make_variant3<LAT, REC, Real, 8, 3, 2, true>();
+        }
+        // tile 15: the paired kernel on the 32 x 16 tile (one CTA per SM)
+        if (tile == 15) {
+            if constexpr (!small_only) return make_variant3<LAT, REC, Real, 16, (f64 ? 2 : 4), 1, true>();
         }
         // tile 10: the paired kernel on 32 x 8 tiles at 2 CTAs/SM (A/B for D3Q27 fp32)
         if (tile == 10) {
@@ -52,6 +61,17 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         // tile 12: split-phase barriers on 32 x 8 tiles at 2 CTAs/SM (A/B, D3Q27 fp32)
         if (tile == 12) {
             if constexpr (!small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true>();
+        }
+        // tiles 13 / 14: one layer body (three rotating accumulator sets), with /
+        // without split-phase barriers, default tile shapes (A/B: I-cache footprint)
+        if (tile == 13 || tile == 14) {
+            if constexpr (LAT == mr::LAT_D3Q19 || small_only) {
+                if (tile == 13) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true, true>();
+                return make_variant3<LAT, REC, Real, 8, 3, 2, true, false, true>();
+            } else {
+                if (tile == 13) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true, true>();
+                return make_variant3<LAT, REC, Real, 8, 3, 2, true, false, true>();
+            }
         }
         if (tile == 9) tile = 0;
         const bool dflt = tile == 0;
