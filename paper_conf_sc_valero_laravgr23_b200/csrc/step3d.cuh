@@ -31,6 +31,10 @@ namespace mr {
 #define MRLBM_Q27_PRODUCT 1
 #endif
 constexpr bool Q27_PRODUCT = MRLBM_Q27_PRODUCT;
+#ifndef MRLBM_ROTATE_PAIRED
+#define MRLBM_ROTATE_PAIRED 0
+#endif
+constexpr bool ROTATE = MRLBM_ROTATE_PAIRED;
 
 // ------------------------------------------------------------ pairs over c_m = (-1, +1)
 template <typename Real> struct Pr;
@@ -645,11 +649,11 @@ __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid
 
     // one layer: on entry X holds layer c-1 and Y layer c; on exit Y holds
     // layer c and Z layer c+1 (Z = X in the two-set scheme)
-    auto layer = [&](const int it, Real (&Xa)[M], Real (&Ya)[M], Real (&Za)[M]) AI {
-        const int c = cfirst + it;
+    // produce(it): collide + reconstruct layer it and publish its c_b != 0 movers
+    // into plane it & 1; the own c_b = 0 row stays in registers (f0, fp)
+    auto produce = [&](const int it, Real (&f0)[3][3], Pr<Real> (&fp)[3][3], Real &rho_own) AI {
         const int s = it % S;
         mbar_wait(&full[s], (it / S) & 1);
-
         Real m[M];
         {
             const Real *st = stage + s * SM::stage_elems + ty * SM::BW + tx + offA;
@@ -659,10 +663,7 @@ __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid
         unsigned char *Fl = planes + (it & 1) * SM::plane_bytes;
         Pr<Real> *Fp = reinterpret_cast<Pr<Real> *>(Fl);
         Real *Fz = reinterpret_cast<Real *>(Fl + size_t(NP) * NT * sizeof(Pr<Real>));
-        // own populations of the c_b = 0 row stay in registers across the barrier
-        Real f0[3][3];
-        Pr<Real> fp[3][3];
-        const Real rho_own = Real(1) + m[0];
+        rho_own = Real(1) + m[0];
         {
             Real A[Basis<LAT, REC>::NH];
             // product form in fp64 only: in fp32 the factors E(c) = w(c) + O(u) round
@@ -688,6 +689,11 @@ __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid
             if constexpr (ps >= 0) Fp[ps * NT + tid] = fp[ca + 1][cb + 1];
             if constexpr (zs >= 0) Fz[zs * NT + tid] = f0[ca + 1][cb + 1];
         });
+    };
+    // the exchange barrier after layer it was published (and the TMA refill of its stage)
+    auto sync_layer = [&](const int it) AI {
+        const int s = it % S;
+        const int c = cfirst + it;
         if constexpr (SPLIT) {
             __syncwarp();
             if (tx == 0) {
@@ -710,6 +716,15 @@ __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid
             }
         }
 
+    };
+    // consume(it): pull layer it from plane it & 1 into the accumulators (X: layer
+    // it - 1, completed and stored; Y: layer it; Z: layer it + 1, started)
+    auto consume = [&](const int it, Real (&Xa)[M], Real (&Ya)[M], Real (&Za)[M], const Real (&f0)[3][3],
+                       const Pr<Real> (&fp)[3][3], const Real rho_own) AI {
+        const int c = cfirst + it;
+        const unsigned char *Fl = planes + (it & 1) * SM::plane_bytes;
+        const Pr<Real> *Fp = reinterpret_cast<const Pr<Real> *>(Fl);
+        const Real *Fz = reinterpret_cast<const Real *>(Fl + size_t(NP) * NT * sizeof(Pr<Real>));
         if (rowlane) {
             const int bbC = (c == 0 && wallClo) ? -1 : ((c == nC - 1 && wallChi) ? 1 : 0);
             auto body = [&](auto open_tag) AI {
@@ -785,12 +800,46 @@ __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid
             }
         }
     };
+    auto layer = [&](const int it, Real (&Xa)[M], Real (&Ya)[M], Real (&Za)[M]) AI {
+        Real f0[3][3];
+        Pr<Real> fp[3][3];
+        Real rho_own;
+        produce(it, f0, fp, rho_own);
+        sync_layer(it);
+        consume(it, Xa, Ya, Za, f0, fp, rho_own);
+    };
     // two accumulator sets with alternating roles (sweep unrolled by two, no
     // accumulator moves) wherever it fits the register file without spills: all
     // but D3Q27 recursive fp64, which keeps three rotating sets
     // ONEBODY: one layer body and three rotating sets (half the loop code: the
     // instruction-cache footprint of the sweep, at 2 M register moves per layer)
-    if constexpr (!ONEBODY && !(LAT == LAT_D3Q27 && REC && sizeof(Real) == 8)) {
+    // ROTATE: the barrier closes each iteration and the block between two barriers
+    // holds the pulls of layer it and the collision + reconstruction of layer
+    // it + 1 -- independent work the compiler interleaves (the FMA-bound synthesis
+    // of one layer overlaps the LSU-bound pulls of the other inside each warp).
+    // Plane it & 1 is read by consume(it) and next written by produce(it + 2),
+    // two barriers later; stage it % S is read by produce(it) before sync_layer(it).
+    if constexpr (ROTATE && !SPLIT && !ONEBODY && !(LAT == LAT_D3Q27 && REC && sizeof(Real) == 8)) {
+        Real f0A[3][3], f0B[3][3];
+        Pr<Real> fpA[3][3], fpB[3][3];
+        Real rA, rB;
+        produce(0, f0A, fpA, rA);
+        sync_layer(0);
+        for (int it = 0; it < nl; it += 2) {
+            if (it + 1 < nl) produce(it + 1, f0B, fpB, rB);
+            consume(it, accA, accB, accA, f0A, fpA, rA);
+            if (it + 1 < nl) {
+                sync_layer(it + 1);
+                if (it + 2 < nl) produce(it + 2, f0A, fpA, rA);
+                consume(it + 1, accB, accA, accB, f0B, fpB, rB);
+                if (it + 2 < nl) sync_layer(it + 2);
+            }
+        }
+        if (owner && clast == c1 - 1) {
+            if (nl & 1) finalize_store(accB, c1 - 1);
+            else finalize_store(accA, c1 - 1);
+        }
+    } else if constexpr (!ONEBODY && !(LAT == LAT_D3Q27 && REC && sizeof(Real) == 8)) {
         for (int it = 0; it < nl; it += 2) {
             layer(it, accA, accB, accA);
             if (it + 1 < nl) layer(it + 1, accB, accA, accB);
