@@ -43,7 +43,7 @@ def needs_build() -> bool:
     return any(p.stat().st_mtime > t for p in DEPS)
 
 
-def build(force: bool = False, verbose: bool = False, out: Path | None = None, defines=()) -> Path:
+def build(force: bool = False, verbose: bool = False, out: Path | None = None, defines=(), extra=()) -> Path:
     """out / defines: a variant build for A/B comparisons (e.g. ab/libmrlbm_X.so, -DNAME)."""
     from concurrent.futures import ThreadPoolExecutor
     import tempfile
@@ -55,7 +55,7 @@ def build(force: bool = False, verbose: bool = False, out: Path | None = None, d
     ncclso = "libnccl.so.2" if (lib / "libnccl.so.2").exists() else "libnccl.so"
     tmp = target.with_suffix(f".{os.getpid()}.tmp.so")
     common = [nvcc(), "-O3", "-std=c++17", *ARCH, "-lineinfo", "--expt-relaxed-constexpr", "-Xcompiler", "-fPIC",
-              f"-I{ROOT / 'include'}", f"-I{inc}", *[f"-D{d}" for d in defines]]
+              f"-I{ROOT / 'include'}", f"-I{inc}", *[f"-D{d}" for d in defines], *extra]
     if verbose:
         common += ["-Xptxas", "-v"]
     with tempfile.TemporaryDirectory(prefix="mrlbm_build_") as td:

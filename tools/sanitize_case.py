@@ -58,5 +58,8 @@ if __name__ == "__main__":
         run("D3Q19", "projective", "fp64", (33, 15, 9), {})
         run("D3Q27", "recursive", "fp32", (33, 31, 9), {"y+": {"kind": "moving_wall", "u": [0.1, 0, 0]},
                                                       "y-": {"kind": "wall"}})
+        # round 3: the paired kernel for D3Q19 fp32 and the product-form D3Q27-R fp64
+        run("D3Q19", "recursive", "fp32", (37, 29, 11), chan3)
+        run("D3Q27", "recursive", "fp64", (33, 19, 9), chan3)
     if which in ("all", "p2p"):
         p2p_pair()
