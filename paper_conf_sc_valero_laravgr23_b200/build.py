@@ -12,9 +12,16 @@ CSRC = PKG / "csrc"
 LIB = PKG / "libmrlbm.so"
 # one translation unit per lattice (compiled in parallel) + the host / ABI unit
 SOURCES = [CSRC / "mrlbm.cu", CSRC / "var_d2q9.cu", CSRC / "var_d3q19.cu", CSRC / "var_d3q27.cu", CSRC / "var_st.cu"]
-DEPS = SOURCES + sorted(CSRC.glob("*.cuh")) + [ROOT / "include" / "mrlbm.h"]
+DEPS = SOURCES + sorted(CSRC.glob("*.cuh")) + [ROOT / "include" / "mrlbm.h", Path(__file__).resolve()]
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+# Per-unit flags.  The D3Q19 unit (the rotated fp64 sweep) is compiled without
+# implicit FMA contraction: its arithmetic spells every fused multiply-add as
+# fma(), so the two halves of the unrolled sweep and the P2P push instance
+# round identically and slab / P2P decompositions stay bitwise equal to one
+# rank (with contraction the compiler fused differently in the two halves:
+# 1-ulp differences; measured cost -0.5% on C5, profiles/r03/ab12.jsonl).
+UNIT_FLAGS = {"var_d3q19.cu": ["-fmad=false"]}
 
 
 def nccl_dirs():
@@ -62,7 +69,9 @@ def build(force: bool = False, verbose: bool = False, out: Path | None = None, d
         objs = [Path(td) / (src.stem + ".o") for src in SOURCES]
 
         def compile_one(i):
-            return subprocess.run(common + ["-c", "-o", str(objs[i]), str(SOURCES[i])], capture_output=True, text=True)
+            flags = UNIT_FLAGS.get(SOURCES[i].name, [])
+            return subprocess.run(common + flags + ["-c", "-o", str(objs[i]), str(SOURCES[i])], capture_output=True,
+                                  text=True)
 
         with ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
             results = list(ex.map(compile_one, range(len(SOURCES))))

@@ -713,7 +713,7 @@ __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> bounce_back(const Real *f
             if (xA) lid(ca < 0 ? 0 : 1);
             if (xB) lid(cb < 0 ? 2 : 3);
             if (xC) lid(cm < 0 ? 4 : 5);
-            v -= Real(wk6) * rho_own * Real(cuw);
+            v = fma(-(Real(wk6) * rho_own), Real(cuw), v); // explicit: same rounding in every instance
             constexpr int ko = X::opp(k);
             if (open) {
                 constexpr int ox = L::c[ko][0], oy = L::c[ko][1];
@@ -777,7 +777,7 @@ __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> finalize_open(RVec<Real, 
                 static_for<q, D>([&](auto rk) {
                     constexpr int r = decltype(rk)::value;
                     constexpr Real H = Real(L::c[k][q] * L::c[k][r]) - ((q == r) ? Real(1.0 / 3.0) : Real(0));
-                    corr[pslot<D>(q, r)] += H * t;
+                    corr[pslot<D>(q, r)] = fma(H, t, corr[pslot<D>(q, r)]);
                 });
             });
         }
@@ -786,8 +786,8 @@ __device__ __forceinline__ RVec<Real, Lattice<LAT>::M> finalize_open(RVec<Real, 
     for (int q = 0; q < D; q++)
 #pragma unroll
         for (int r = q; r < D; r++)
-            out.v[pslot<D>(q, r)] = s.v[pslot<D>(q, r)] - ((q == r) ? S0 * Real(1.0 / 3.0) : Real(0)) -
-                                    Real(6) * rho * corr[pslot<D>(q, r)];
+            out.v[pslot<D>(q, r)] = fma(Real(-6) * rho, corr[pslot<D>(q, r)],
+                                        (q == r) ? fma(S0, Real(-1.0 / 3.0), s.v[pslot<D>(q, r)]) : s.v[pslot<D>(q, r)]);
     return out;
 }
 
@@ -1004,7 +1004,7 @@ __global__ void __launch_bounds__(TA *TB, MINB) mrlbm_step_kernel(const __grid_c
             for (int q = 0; q < D; q++)
 #pragma unroll
                 for (int r = q; r < D; r++)
-                    out[pslot<D>(q, r)] = s[pslot<D>(q, r)] - ((q == r) ? S0 * Real(1.0 / 3.0) : Real(0));
+                    out[pslot<D>(q, r)] = (q == r) ? fma(S0, Real(-1.0 / 3.0), s[pslot<D>(q, r)]) : s[pslot<D>(q, r)];
         } else {
             RVec<Real, M> sv;
 #pragma unroll

@@ -612,7 +612,7 @@ __global__ void __launch_bounds__(32 * TB, MINB) mrlbm_step3_kernel(const __grid
             for (int q = 0; q < 3; q++)
 #pragma unroll
                 for (int r = q; r < 3; r++)
-                    out[pslot<3>(q, r)] = s[pslot<3>(q, r)] - ((q == r) ? S0 * Real(1.0 / 3.0) : Real(0));
+                    out[pslot<3>(q, r)] = (q == r) ? fma(S0, Real(-1.0 / 3.0), s[pslot<3>(q, r)]) : s[pslot<3>(q, r)];
         } else {
             RVec<Real, M> sv;
 #pragma unroll

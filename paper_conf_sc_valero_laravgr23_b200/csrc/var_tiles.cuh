@@ -45,6 +45,10 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         if (tile == 0 && cluster != 2) {
             if constexpr (LAT == mr::LAT_D3Q27 || !f64) return make_variant3<LAT, REC, Real, 8, 3, 2, true>();
         }
+        // tile 16: the paired kernel on 32 x 8 tiles with a 5-deep TMA ring (fp32 fits at 2 CTAs/SM)
+        if (tile == 16) {
+            if constexpr (!f64) return make_variant3<LAT, REC, Real, 8, 5, 2, true>();
+        }
         // tile 15: the paired kernel on the 32 x 16 tile (one CTA per SM)
         if (tile == 15) {
             if constexpr (!small_only) return make_variant3<LAT, REC, Real, 16, (f64 ? 2 : 4), 1, true>();
