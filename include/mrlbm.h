@@ -132,7 +132,9 @@ typedef int mrlbm_status;
 #define MRLBM_OK 0
 #define MRLBM_ERR_INVALID_ARGUMENT -1 /* tau <= 1/2, n < 2, D2Q9 with nz != 1, one-sided periodic, bad kind */
 #define MRLBM_ERR_UNSUPPORTED -2      /* open faces sharing an edge, open face on the marching axis;
-                                         BGK with MOMENTS; DISTRIBUTIONS with open faces or nranks > 1 */
+                                         BGK with MOMENTS; DISTRIBUTIONS with open faces or nranks > 1;
+                                         a layer of M * (ny + 2) * pitch >= 2^31 elements (3D in-plane
+                                         sizes beyond ~14000^2: the step kernels use 32-bit offsets) */
 #define MRLBM_ERR_OUT_OF_MEMORY -3
 #define MRLBM_ERR_CUDA -4
 #define MRLBM_ERR_NCCL -5
