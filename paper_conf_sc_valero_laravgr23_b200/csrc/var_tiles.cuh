@@ -17,14 +17,8 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
     if constexpr (LAT == mr::LAT_D2Q9) {
         (void)cluster;
         // deeper TMA rings trade resident CTAs for bytes in flight (tuning: MRLBM_TILE)
+        // (the round-2 ring-depth sweep variants 2..7 are retired: profiles/ring2d_*_r02.jsonl)
         if (tile == 1) return make_variant<LAT, REC, Real, 128, 1, 4, 4>();
-        if (tile == 2) return make_variant<LAT, REC, Real, 128, 1, 6, 4>();
-        if (tile == 3) return make_variant<LAT, REC, Real, 128, 1, 8, 3>();
-        // fp32: a stage is only 3 KB, so deep rings fit at 5 CTAs per SM
-        if (tile == 4) return make_variant<LAT, REC, Real, 128, 1, 8, 5>();
-        if (tile == 5) return make_variant<LAT, REC, Real, 128, 1, 12, 5>();
-        if (tile == 6) return make_variant<LAT, REC, Real, 128, 1, 5, 4>();
-        if (tile == 7) return make_variant<LAT, REC, Real, 128, 1, 6, 6>();
         if (tile == 8) return make_variant<LAT, REC, Real, 128, 1, 4, 5>(); // round-1 default
         // default: a 6-deep TMA ring; fp64 at 4 CTAs/SM (6 x 6.2 KB stages), fp32 at 6
         // (measured C2: fp64 0.90 -> 0.916, fp32 0.80 -> 0.82; profiles/ring2d_b_r02.jsonl)
@@ -45,10 +39,6 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         if (tile == 0 && cluster != 2) {
             if constexpr (LAT == mr::LAT_D3Q27 || !f64) return make_variant3<LAT, REC, Real, 8, 3, 2, true>();
         }
-        // tile 16: the paired kernel on 32 x 8 tiles with a 5-deep TMA ring (fp32 fits at 2 CTAs/SM)
-        if (tile == 16) {
-            if constexpr (!f64) return make_variant3<LAT, REC, Real, 8, 5, 2, true>();
-        }
         // tile 15: the paired kernel on the 32 x 16 tile (one CTA per SM)
         if (tile == 15) {
             if constexpr (!small_only) return make_variant3<LAT, REC, Real, 16, (f64 ? 2 : 4), 1, true>();
@@ -57,26 +47,9 @@ template <int LAT, bool REC, typename Real> Variant pick(int tile, int cluster)
         if (tile == 10) {
             if constexpr (!small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true>();
         }
-        // tile 11: the paired kernel with split-phase exchange barriers (A/B)
-        if (tile == 11) {
-            if constexpr (LAT == mr::LAT_D3Q19 || small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true>();
-            else return make_variant3<LAT, REC, Real, 16, (f64 ? 2 : 4), 1, true, true>();
-        }
-        // tile 12: split-phase barriers on 32 x 8 tiles at 2 CTAs/SM (A/B, D3Q27 fp32)
-        if (tile == 12) {
-            if constexpr (!small_only) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true>();
-        }
-        // tiles 13 / 14: one layer body (three rotating accumulator sets), with /
-        // without split-phase barriers, default tile shapes (A/B: I-cache footprint)
-        if (tile == 13 || tile == 14) {
-            if constexpr (LAT == mr::LAT_D3Q19 || small_only) {
-                if (tile == 13) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true, true>();
-                return make_variant3<LAT, REC, Real, 8, 3, 2, true, false, true>();
-            } else {
-                if (tile == 13) return make_variant3<LAT, REC, Real, 8, 3, 2, true, true, true>();
-                return make_variant3<LAT, REC, Real, 8, 3, 2, true, false, true>();
-            }
-        }
+        // (round-3 A/B variants retired after measurement, profiles/r03/: tile 11/12
+        // split-phase barriers, 13/14 one-body sweeps, 16 a 5-deep paired ring; the
+        // kernel keeps the SPLIT / ONEBODY template options)
         if (tile == 9) tile = 0;
         const bool dflt = tile == 0;
         if (tile == 0) tile = (LAT == mr::LAT_D3Q19 || small_only) ? 1 : 2;
