@@ -670,10 +670,12 @@ mrlbm_status mrlbm_create(mrlbm_t *out, mrlbm_lattice lattice, int64_t nx, int64
     h->tilesB = h->D == 3 ? (h->nB + CL * TB - 3) / (CL * TB - 2) * CL : 1;
     a.tilesA = h->tilesA;
     a.tilesB = h->tilesB;
-    // 3D launch order: groups of MRLBM_RAST B-tiles (tuning; default 0 = the plain
-    // (A, B) grid: measured C3 -2% / -5% at groups of 4 / 8, C5 +0.6%, C4 -0.3%,
-    // profiles/ab_r03.md)
-    a.rastG = (h->D == 3 && CL == 1) ? std::max(0, env_int("MRLBM_RAST", 0)) : 0;
+    // 3D launch order: groups of MRLBM_RAST B-tiles.  Default: groups of 4 on wide
+    // planes (>= 32 tiles along A, where B-neighbour tiles launched tilesA CTAs apart
+    // no longer meet in L2: C5w DRAM reads 14.9 -> 13.6 GB per step, +0.3%), the
+    // plain (A, B) grid otherwise (C3: groups cost 0.7-5%); profiles/r03/ab1.jsonl, ab14.jsonl
+    const int rast_default = h->tilesA >= 32 ? 4 : 0;
+    a.rastG = (h->D == 3 && CL == 1) ? std::max(0, env_int("MRLBM_RAST", rast_default)) : 0;
     // Segments along C.  The grid is tiles x segments; pick the segment count
     // that best fills whole waves of resident CTAs (no tail wave), preferring
     // longer segments (each segment re-reads one halo layer at each end).
